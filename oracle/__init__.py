@@ -1,0 +1,103 @@
+"""oracle -- TEST INFRASTRUCTURE ONLY.
+
+A plain, slow, obviously correct CPU implementation of what the CUDA path of
+paper_conf_spaa_berneys25_b200 computes, written from the paper
+(/root/reference/PAPER.md, cited as PAPER.md:<line>):
+
+    sort_oracle.c   stable top-down mergesort: u32, f32 (IEEE totalOrder), pairs
+    addrmap.py      pi, rho and Alg. 1's gather schedule (§3)
+    dmm.py          DMM bank-conflict cost model + Thrust serial-merge address stream
+    worstcase.py    Section 4 worst-case construction (S, T, Theorem 8) + composition
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+`--impl reference` leg may import, call, link or execute anything under
+oracle/.  The product path never does, and the oracle never imports the
+product package: the two share only `synthetic_inputs` (seeded generators,
+none of the method's arithmetic).
+
+Parity status of each function is listed in DESIGN.md §"Oracle and pins"; every
+function here is pinned by tests/test_oracle_*.py to something other than
+itself (library routines, brute force, the paper's figures and closed forms).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "sort_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile sort_oracle.c with gcc (plain C, -O2, single thread)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(
+            ["gcc", "-O2", "-std=c99", "-shared", "-fPIC", "-o", _LIB, _SRC]
+        )
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB)
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        for name in ("oracle_sort_u32", "oracle_sort_f32"):
+            f = getattr(L, name)
+            f.argtypes = [u32p, u32p, ctypes.c_uint64]
+            f.restype = ctypes.c_int
+        L.oracle_sort_pairs_u32.argtypes = [u32p, u32p, u32p, u32p, ctypes.c_uint64]
+        L.oracle_sort_pairs_u32.restype = ctypes.c_int
+        L.oracle_f32_total_less.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
+        L.oracle_f32_total_less.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
+
+
+def sort_u32(keys: np.ndarray) -> np.ndarray:
+    k = np.ascontiguousarray(keys, dtype=np.uint32)
+    out = np.empty_like(k)
+    if lib().oracle_sort_u32(_p(k), _p(out), k.size) != 0:
+        raise MemoryError("oracle_sort_u32")
+    return out
+
+
+def sort_f32_bits(bits: np.ndarray) -> np.ndarray:
+    """Keys given and returned as uint32 bit patterns of binary32 floats."""
+    k = np.ascontiguousarray(bits, dtype=np.uint32)
+    out = np.empty_like(k)
+    if lib().oracle_sort_f32(_p(k), _p(out), k.size) != 0:
+        raise MemoryError("oracle_sort_f32")
+    return out
+
+
+def sort_pairs_u32(keys: np.ndarray, vals: np.ndarray):
+    k = np.ascontiguousarray(keys, dtype=np.uint32)
+    v = np.ascontiguousarray(vals, dtype=np.uint32)
+    assert k.size == v.size
+    ko = np.empty_like(k)
+    vo = np.empty_like(v)
+    if lib().oracle_sort_pairs_u32(_p(k), _p(v), _p(ko), _p(vo), k.size) != 0:
+        raise MemoryError("oracle_sort_pairs_u32")
+    return ko, vo
+
+
+def f32_total_less(a: int, b: int) -> bool:
+    return bool(lib().oracle_f32_total_less(a & 0xFFFFFFFF, b & 0xFFFFFFFF))
+
+
+def dist_rank_slice(sorted_global: np.ndarray, rank: int, world: int):
+    """Rank r of an exactly balanced distributed sort holds positions
+    [floor(r n / p), floor((r+1) n / p)) of the global stable order."""
+    n = sorted_global.shape[0]
+    return sorted_global[(rank * n) // world:((rank + 1) * n) // world]
