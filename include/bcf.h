@@ -1,0 +1,149 @@
+/*
+ * bcf.h -- C ABI of the B200-native bank-conflict-free mergesort.
+ *
+ * Implements the hot path of K. Berney, N. Sitchinava, "Eliminating Bank
+ * Conflicts in GPU Mergesort", SPAA '25 (cited as PAPER.md:<line>):
+ * Thrust-style stable pairwise mergesort (PAPER.md:59-61 §1, :348-354 §5)
+ * whose shared-memory tiles use the paper's permutation rho(A u pi(B))
+ * (Alg. 1 line 2; §3.1-3.3) and the load-balanced dual
+ * subsequence gather (Alg. 1), so that no input causes a
+ * shared-memory bank conflict.
+ *
+ * Conventions (all entry points):
+ *  - Pointers named d_* are DEVICE pointers (cudaMalloc / torch CUDA tensors)
+ *    on the current device; h_* are HOST pointers.  The caller owns all
+ *    memory; the library never allocates device memory.
+ *  - Temporary storage is queried CUB-style: call with d_temp == NULL to get
+ *    *temp_bytes, then call again with a buffer of at least that size.
+ *  - All device work is enqueued on `stream` (may be 0 = legacy default
+ *    stream) and is asynchronous; nothing synchronizes the host, except
+ *    bcf_worst_case_u32 (host-built input, copied with a synchronous H2D) and
+ *    bcf_profile_collect.
+ *  - Argument errors are returned synchronously before any launch.
+ *    n > 0 with a NULL data pointer -> BCF_ERROR_INVALID_VALUE; a temp buffer
+ *    smaller than required -> BCF_ERROR_TEMP_TOO_SMALL; (E, u) outside the
+ *    instantiated set -> BCF_ERROR_UNSUPPORTED.  Launch / runtime errors
+ *    return BCF_ERROR_CUDA and bcf_last_cuda_error() gives the cudaError_t
+ *    (thread-local).  No C++ exception crosses this boundary.
+ *  - n = 0 is a no-op; d_in == d_out (in place) is allowed.
+ *  - n is 64-bit; sizes up to 2^32 keys are supported (bounded by memory).
+ *  - Thread-safe: no mutable global state except the optional profiler.
+ */
+#ifndef BCF_H_
+#define BCF_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BCF_ABI_VERSION 1
+
+typedef enum {
+  BCF_SUCCESS = 0,
+  BCF_ERROR_INVALID_VALUE = 1,
+  BCF_ERROR_UNSUPPORTED = 2,
+  BCF_ERROR_CUDA = 3,
+  BCF_ERROR_TEMP_TOO_SMALL = 4
+} bcf_status;
+
+typedef enum {
+  /* the paper's bank-conflict-free design (CF-Merge) */
+  BCF_ALGO_CONFLICT_FREE = 0,
+  /* the unmodified Thrust design the paper compares against (A|B forward in
+     shared memory, per-thread merge-path binary search, serial merge reading
+     shared memory).  Keys only (u32 / f32). */
+  BCF_ALGO_BASELINE = 1
+} bcf_algo;
+
+/* "software parameters" E and u: items per thread and threads
+   per block.  0 selects the default.  Instantiated set: E in [7, 17],
+   u in {128, 256, 512}. */
+typedef struct {
+  int32_t items_per_thread; /* E */
+  int32_t block_threads;    /* u */
+  int32_t algo;             /* bcf_algo */
+} bcf_params;
+
+/* Default (E, u) chosen for sm_100a. */
+void bcf_default_params(bcf_params* p);
+
+/* Stable sort of n u32 keys, ascending ("4-byte
+   integers").  d_in is not modified unless d_in == d_out.
+   Temp: n keys (+ alignment).  p may be NULL (defaults). */
+bcf_status bcf_sort_u32(const uint32_t* d_in, uint32_t* d_out, uint64_t n, void* d_temp,
+                        size_t* temp_bytes, const bcf_params* p, void* stream);
+
+/* Sort n f32 keys by IEEE 754 totalOrder (-NaN < -inf < ... < -0 < +0 < ...
+   < +inf < +NaN; reading c2).  Keys are encoded to order-preserving
+   u32 on the first load and decoded on the final store (fused, no extra
+   pass).  Ties are bit-identical, so stability is unobservable. */
+bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_temp,
+                        size_t* temp_bytes, const bcf_params* p, void* stream);
+
+/* Stable sort of (key, value) pairs by u32 key; values (u32) follow their
+   keys; equal keys keep their input order.  Temp: n keys + n values.
+   BCF_ALGO_BASELINE is not supported for pairs (BCF_ERROR_UNSUPPORTED). */
+bcf_status bcf_sort_pairs_u32(const uint32_t* d_keys_in, uint32_t* d_keys_out,
+                              const uint32_t* d_vals_in, uint32_t* d_vals_out, uint64_t n,
+                              void* d_temp, size_t* temp_bytes, const bcf_params* p, void* stream);
+
+/* Worst-case input for the unmodified Thrust mergesort with parameters
+   (E, u) (Section 4: sequences S and T, Theorem 8;
+   multi-level composition per DESIGN.md reading c10).  Writes a permutation
+   of 0..n-1 to d_out.  Deterministic in (n, E, u, seed).  Host-built, then a
+   synchronous copy to the device (off the timed path).  E in [2, 32]. */
+bcf_status bcf_worst_case_u32(uint32_t* d_out, uint64_t n, int32_t E, int32_t u, uint64_t seed,
+                              void* stream);
+/* Same construction into host memory (no CUDA call). */
+bcf_status bcf_worst_case_u32_host(uint32_t* h_out, uint64_t n, int32_t E, int32_t u,
+                                   uint64_t seed);
+
+/* Distributed-sort phases (the exchange itself is done by torch.distributed).
+   For each of npiv pivots v (device array), count the keys of the sorted
+   run d_sorted[0, n) that are < v and <= v (binary searches, one thread per
+   pivot).  Outputs are device arrays of npiv u64. */
+bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint32_t* d_pivots,
+                                int32_t npiv, uint64_t* d_lt_counts, uint64_t* d_le_counts,
+                                void* stream);
+
+/* Stable merge of nruns ascending sorted runs stored back to back in d_runs
+   (run r = [h_run_offsets[r], h_run_offsets[r+1]), host array of nruns+1
+   entries, h_run_offsets[0] = 0); equal keys keep run order (run 0 first).
+   Output ascending in d_out (must not alias d_runs).  Pairwise passes of the
+   same CF merge kernel.  Values: pass NULL for keys only. */
+bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals,
+                              const uint64_t* h_run_offsets, int32_t nruns, uint32_t* d_out,
+                              uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes,
+                              const bcf_params* p, void* stream);
+
+const char* bcf_status_string(bcf_status s);
+int32_t bcf_abi_version(void);
+/* cudaError_t (as int) of the last BCF_ERROR_CUDA on the calling thread */
+int32_t bcf_last_cuda_error(void);
+
+/* ---- measurement hooks (bench.py) ----------------------------------------
+   When enabled, every kernel launched by the library is bracketed by CUDA
+   events recorded on the launch stream; bcf_profile_collect synchronizes
+   those events and returns, per kernel class, the number of launches and the
+   summed device milliseconds.  Disabled by default (zero overhead). */
+typedef struct {
+  char name[32];     /* "block_sort", "merge_pass", "split_counts", ... */
+  int64_t launches;
+  double total_ms;
+  uint64_t keys;     /* keys processed by those launches (sum of n) */
+} bcf_kernel_stats;
+
+bcf_status bcf_profile_enable(int32_t on);
+/* fills up to max entries, *count = number of classes; resets the record */
+bcf_status bcf_profile_collect(bcf_kernel_stats* out, int32_t max, int32_t* count);
+/* total kernels launched by this process through the library (always on) */
+int64_t bcf_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* BCF_H_ */

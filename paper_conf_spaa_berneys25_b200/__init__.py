@@ -1,0 +1,260 @@
+"""paper_conf_spaa_berneys25_b200 -- B200-native bank-conflict-free mergesort.
+
+Thin Python binding over the C ABI in include/bcf.h (libbcf.so, built
+in-tree for sm_100a).  Argument marshalling only: every step of the sort runs
+in the library's CUDA kernels.  PyTorch provides device memory and streams.
+There is no CPU fallback: without the extension or without a CUDA tensor the
+calls raise.
+
+    sort(keys)                 u32 / i32 (as u32 bit patterns) / f32 (totalOrder)
+    sort_pairs(keys, values)   stable by u32 key
+    worst_case(n, E, u, seed)  Section 4 worst-case permutation (device tensor)
+    worst_case_host(...)       same into a numpy array (no CUDA)
+    split_counts, merge_runs   distributed-sort phases (see dist.py)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbcf.so")
+
+BCF_SUCCESS = 0
+BCF_ERROR_INVALID_VALUE = 1
+BCF_ERROR_UNSUPPORTED = 2
+BCF_ERROR_CUDA = 3
+BCF_ERROR_TEMP_TOO_SMALL = 4
+ALGO_CONFLICT_FREE = 0
+ALGO_BASELINE = 1
+
+# every symbol include/bcf.h declares
+EXPORTED_SYMBOLS = [
+    "bcf_default_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
+    "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
+    "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
+    "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count",
+]
+
+
+class BcfError(RuntimeError):
+    pass
+
+
+class Params(ctypes.Structure):
+    _fields_ = [("items_per_thread", ctypes.c_int32), ("block_threads", ctypes.c_int32),
+                ("algo", ctypes.c_int32)]
+
+
+class KernelStats(ctypes.Structure):
+    _fields_ = [("name", ctypes.c_char * 32), ("launches", ctypes.c_int64),
+                ("total_ms", ctypes.c_double), ("keys", ctypes.c_uint64)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libbcf.so (raises if it was not built: run build() first)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise BcfError(f"{LIB_PATH} missing: build it with paper_conf_spaa_berneys25_b200.build.build()")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, sz = ctypes.c_void_p, ctypes.c_size_t
+    u64, i32 = ctypes.c_uint64, ctypes.c_int32
+    P = ctypes.POINTER
+    L.bcf_default_params.argtypes = [P(Params)]
+    L.bcf_default_params.restype = None
+    for name in ("bcf_sort_u32", "bcf_sort_f32"):
+        f = getattr(L, name)
+        f.argtypes = [vp, vp, u64, vp, P(sz), P(Params), vp]
+        f.restype = ctypes.c_int
+    L.bcf_sort_pairs_u32.argtypes = [vp, vp, vp, vp, u64, vp, P(sz), P(Params), vp]
+    L.bcf_sort_pairs_u32.restype = ctypes.c_int
+    L.bcf_worst_case_u32.argtypes = [vp, u64, i32, i32, u64, vp]
+    L.bcf_worst_case_u32.restype = ctypes.c_int
+    L.bcf_worst_case_u32_host.argtypes = [vp, u64, i32, i32, u64]
+    L.bcf_worst_case_u32_host.restype = ctypes.c_int
+    L.bcf_split_counts_u32.argtypes = [vp, u64, vp, i32, vp, vp, vp]
+    L.bcf_split_counts_u32.restype = ctypes.c_int
+    L.bcf_merge_runs_u32.argtypes = [vp, vp, P(u64), i32, vp, vp, vp, P(sz), P(Params), vp]
+    L.bcf_merge_runs_u32.restype = ctypes.c_int
+    L.bcf_status_string.argtypes = [ctypes.c_int]
+    L.bcf_status_string.restype = ctypes.c_char_p
+    L.bcf_abi_version.restype = i32
+    L.bcf_last_cuda_error.restype = i32
+    L.bcf_profile_enable.argtypes = [i32]
+    L.bcf_profile_enable.restype = ctypes.c_int
+    L.bcf_profile_collect.argtypes = [P(KernelStats), i32, P(i32)]
+    L.bcf_profile_collect.restype = ctypes.c_int
+    L.bcf_launch_count.restype = ctypes.c_int64
+    _lib = L
+    return L
+
+
+def _check(st: int, what: str):
+    if st != BCF_SUCCESS:
+        msg = lib().bcf_status_string(st).decode()
+        if st == BCF_ERROR_CUDA:
+            msg += f" (cudaError {lib().bcf_last_cuda_error()})"
+        raise BcfError(f"{what}: {msg}")
+
+
+def default_params() -> Params:
+    p = Params()
+    lib().bcf_default_params(ctypes.byref(p))
+    return p
+
+
+def make_params(E: int = 0, u: int = 0, algo: int = ALGO_CONFLICT_FREE) -> Params:
+    return Params(E, u, algo)
+
+
+def _torch():
+    import torch
+
+    return torch
+
+
+def _require_cuda(t, name):
+    torch = _torch()
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise BcfError(f"{name} must be a CUDA tensor (no CPU path)")
+    if not t.is_contiguous():
+        raise BcfError(f"{name} must be contiguous")
+    if t.element_size() != 4:
+        raise BcfError(f"{name} must have 4-byte elements")
+
+
+def _stream(t):
+    torch = _torch()
+    return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
+
+
+def _temp(nbytes: int, device):
+    torch = _torch()
+    return torch.empty(max(1, int(nbytes)), dtype=torch.uint8, device=device)
+
+
+def sort(keys, out=None, params: Params | None = None, temp=None):
+    """Sort a 1-D CUDA tensor of 4-byte keys.  float32: IEEE totalOrder;
+    int32 / uint32: keys are sorted as unsigned 32-bit bit patterns."""
+    torch = _torch()
+    _require_cuda(keys, "keys")
+    n = keys.numel()
+    if out is None:
+        out = torch.empty_like(keys)
+    _require_cuda(out, "out")
+    is_f32 = keys.dtype == torch.float32
+    fn = lib().bcf_sort_f32 if is_f32 else lib().bcf_sort_u32
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    _check(fn(None, None, n, None, ctypes.byref(tb), pp, None), "temp query")
+    if temp is None or temp.numel() < tb.value:
+        temp = _temp(tb.value, keys.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(keys.device):
+        _check(fn(keys.data_ptr(), out.data_ptr(), n, temp.data_ptr(), ctypes.byref(tb), pp,
+                  _stream(keys)), "bcf_sort")
+    return out
+
+
+def sort_pairs(keys, values, keys_out=None, values_out=None, params: Params | None = None, temp=None):
+    torch = _torch()
+    _require_cuda(keys, "keys")
+    _require_cuda(values, "values")
+    n = keys.numel()
+    if values.numel() != n:
+        raise BcfError("keys and values differ in length")
+    keys_out = torch.empty_like(keys) if keys_out is None else keys_out
+    values_out = torch.empty_like(values) if values_out is None else values_out
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    L = lib()
+    _check(L.bcf_sort_pairs_u32(None, None, None, None, n, None, ctypes.byref(tb), pp, None), "temp query")
+    if temp is None or temp.numel() < tb.value:
+        temp = _temp(tb.value, keys.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(keys.device):
+        _check(L.bcf_sort_pairs_u32(keys.data_ptr(), keys_out.data_ptr(), values.data_ptr(),
+                                    values_out.data_ptr(), n, temp.data_ptr(), ctypes.byref(tb), pp,
+                                    _stream(keys)), "bcf_sort_pairs_u32")
+    return keys_out, values_out
+
+
+def worst_case(n: int, E: int, u: int, seed: int = 0, device="cuda"):
+    torch = _torch()
+    out = torch.empty(n, dtype=torch.int32, device=device)
+    with torch.cuda.device(out.device):
+        _check(lib().bcf_worst_case_u32(out.data_ptr() if n else None, n, E, u, seed & (2**64 - 1),
+                                        _stream(out)), "bcf_worst_case_u32")
+    return out
+
+
+def worst_case_host(n: int, E: int, u: int, seed: int = 0) -> np.ndarray:
+    out = np.empty(n, dtype=np.uint32)
+    _check(lib().bcf_worst_case_u32_host(out.ctypes.data if n else None, n, E, u, seed & (2**64 - 1)),
+           "bcf_worst_case_u32_host")
+    return out
+
+
+def split_counts(sorted_keys, pivots):
+    """(lt, le) counts of each pivot in a sorted CUDA run (int64 tensors)."""
+    torch = _torch()
+    _require_cuda(sorted_keys, "sorted_keys")
+    _require_cuda(pivots, "pivots")
+    lt = torch.empty(pivots.numel(), dtype=torch.int64, device=sorted_keys.device)
+    le = torch.empty_like(lt)
+    with torch.cuda.device(sorted_keys.device):
+        _check(lib().bcf_split_counts_u32(sorted_keys.data_ptr(), sorted_keys.numel(), pivots.data_ptr(),
+                                          pivots.numel(), lt.data_ptr(), le.data_ptr(),
+                                          _stream(sorted_keys)), "bcf_split_counts_u32")
+    return lt, le
+
+
+def merge_runs(runs, run_offsets, values=None, params: Params | None = None):
+    """Stable merge of ascending runs stored back to back (run order breaks ties)."""
+    torch = _torch()
+    _require_cuda(runs, "runs")
+    offs = np.ascontiguousarray(np.asarray(run_offsets, dtype=np.uint64))
+    nruns = len(offs) - 1
+    out = torch.empty_like(runs)
+    out_v = torch.empty_like(values) if values is not None else None
+    L = lib()
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    optr = offs.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))
+    vptr = values.data_ptr() if values is not None else None
+    _check(L.bcf_merge_runs_u32(runs.data_ptr(), vptr, optr, nruns, None, None, None, ctypes.byref(tb), pp,
+                                None), "temp query")
+    temp = _temp(tb.value, runs.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(runs.device):
+        _check(L.bcf_merge_runs_u32(runs.data_ptr(), vptr, optr, nruns, out.data_ptr(),
+                                    out_v.data_ptr() if out_v is not None else None, temp.data_ptr(),
+                                    ctypes.byref(tb), pp, _stream(runs)), "bcf_merge_runs_u32")
+    return (out, out_v) if values is not None else out
+
+
+def profile_enable(on: bool = True):
+    _check(lib().bcf_profile_enable(1 if on else 0), "bcf_profile_enable")
+
+
+def profile_collect() -> dict:
+    arr = (KernelStats * 32)()
+    cnt = ctypes.c_int32(0)
+    _check(lib().bcf_profile_collect(arr, 32, ctypes.byref(cnt)), "bcf_profile_collect")
+    return {arr[i].name.decode(): {"launches": arr[i].launches, "total_ms": arr[i].total_ms,
+                                   "keys": arr[i].keys} for i in range(cnt.value)}
+
+
+def launch_count() -> int:
+    return int(lib().bcf_launch_count())
+
+
+def abi_version() -> int:
+    return int(lib().bcf_abi_version())

@@ -1,0 +1,392 @@
+// bcf_capi.cu -- the C ABI (include/bcf.h): argument checking, the pass
+// driver of the pairwise mergesort, temp sizing,
+// launch dispatch over the instantiated (E, u) set, the distributed-sort
+// helper kernels and the optional per-kernel event profiler.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/bcf.h"
+#include "bcf_kernels.cuh"
+#include "bcf_launch.h"
+
+namespace bcf {
+namespace wc {
+void generate(uint32_t* out, uint64_t n, int E, int u, uint64_t seed);
+}
+
+// ---------------------------------------------------------------------------
+// launch table
+// ---------------------------------------------------------------------------
+LaunchTable& launch_table() {
+  static LaunchTable* t = [] {
+    auto* p = new LaunchTable();
+    register_E7(*p);
+    register_E8(*p);
+    register_E9(*p);
+    register_E10(*p);
+    register_E11(*p);
+    register_E12(*p);
+    register_E13(*p);
+    register_E14(*p);
+    register_E15(*p);
+    register_E16(*p);
+    register_E17(*p);
+    return p;
+  }();
+  return *t;
+}
+
+// Defaults for sm_100a: E = 16 makes the in-register
+// merge a pure 16-wide bitonic merger (no rotation) and the tile a power of
+// two; rho (d = 16) keeps every shared-memory access conflict-free.
+static constexpr int DEFAULT_E = 16;
+static constexpr int DEFAULT_U = 256;
+
+// ---------------------------------------------------------------------------
+// errors, profiler, launch accounting
+// ---------------------------------------------------------------------------
+static thread_local int t_last_cuda_error = 0;
+static std::atomic<long long> g_launches{0};
+static std::atomic<int> g_prof_on{0};
+static std::mutex g_prof_mu;
+
+struct ProfRec {
+  const char* name;
+  cudaEvent_t a, b;
+  uint64_t keys;
+};
+static std::vector<ProfRec> g_recs;
+static std::vector<cudaEvent_t> g_pool;
+
+static cudaEvent_t pool_get() {
+  cudaEvent_t e = nullptr;
+  if (!g_pool.empty()) {
+    e = g_pool.back();
+    g_pool.pop_back();
+    return e;
+  }
+  cudaEventCreate(&e);
+  return e;
+}
+
+static bcf_status cuda_fail(cudaError_t e) {
+  t_last_cuda_error = (int)e;
+  return BCF_ERROR_CUDA;
+}
+
+template <class F>
+static cudaError_t launch(const char* name, uint64_t keys, cudaStream_t s, F&& f) {
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  if (!g_prof_on.load(std::memory_order_relaxed)) return f();
+  cudaEvent_t a, b;
+  {
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    a = pool_get();
+    b = pool_get();
+  }
+  cudaEventRecord(a, s);
+  cudaError_t e = f();
+  cudaEventRecord(b, s);
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  g_recs.push_back({name, a, b, keys});
+  return e;
+}
+
+struct Params {
+  int E, U, algo;
+};
+
+static bcf_status resolve(const bcf_params* p, Params& out) {
+  out.E = (p && p->items_per_thread) ? p->items_per_thread : DEFAULT_E;
+  out.U = (p && p->block_threads) ? p->block_threads : DEFAULT_U;
+  out.algo = p ? p->algo : BCF_ALGO_CONFLICT_FREE;
+  if (out.algo != BCF_ALGO_CONFLICT_FREE && out.algo != BCF_ALGO_BASELINE) return BCF_ERROR_INVALID_VALUE;
+  if (out.E < E_MIN || out.E > E_MAX || u_index(out.U) < 0) return BCF_ERROR_UNSUPPORTED;
+  return BCF_SUCCESS;
+}
+
+static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// ---------------------------------------------------------------------------
+// the pairwise mergesort driver
+//   block sort: tiles of T = U*E -> runs of T (run r descending iff r odd, CF)
+//   pass i = 1..P: runs of R = T*2^(i-1) merged pairwise; pass P writes d_out
+// buffers: buf[0] = out, buf[1] = temp; the block sort writes buf[P % 2] and
+// pass i writes buf[(P - i) % 2], so the last pass lands in out.
+// ---------------------------------------------------------------------------
+static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_t* in_v, uint32_t* out_v,
+                            uint64_t n, void* d_temp, size_t* temp_bytes, const bcf_params* pp,
+                            cudaStream_t s, bool f32, bool pairs) {
+  if (!temp_bytes) return BCF_ERROR_INVALID_VALUE;
+  Params p;
+  bcf_status st = resolve(pp, p);
+  if (st != BCF_SUCCESS) return st;
+  if (pairs && p.algo == BCF_ALGO_BASELINE) return BCF_ERROR_UNSUPPORTED;
+  const size_t key_bytes = align_up((size_t)n * sizeof(uint32_t), 256);
+  const size_t need = 256 + key_bytes * (pairs ? 2 : 1);
+  if (d_temp == nullptr) {
+    *temp_bytes = need;
+    return BCF_SUCCESS;
+  }
+  if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
+  if (n == 0) return BCF_SUCCESS;
+  if (!in_k || !out_k || (pairs && (!in_v || !out_v))) return BCF_ERROR_INVALID_VALUE;
+  if (n > (1ull << 33)) return BCF_ERROR_UNSUPPORTED;
+
+  const Variant& var = launch_table().v[p.E][u_index(p.U)][p.algo][pairs ? 1 : 0];
+  if (!var.block_sort || !var.merge) return BCF_ERROR_UNSUPPORTED;
+  const long long T = (long long)p.U * p.E;
+  const long long tiles = (long long)((n + T - 1) / T);
+  int P = 0;
+  while ((T << P) < (long long)n) ++P;
+  const bool cf = p.algo == BCF_ALGO_CONFLICT_FREE;
+
+  char* tb = (char*)align_up((size_t)d_temp, 256);
+  uint32_t* tk = (uint32_t*)tb;
+  uint32_t* tv = pairs ? (uint32_t*)(tb + key_bytes) : nullptr;
+  uint32_t* bk[2] = {out_k, tk};
+  uint32_t* bv[2] = {out_v, tv};
+
+  SortArgs sa{in_k, in_v, bk[P % 2], bv[P % 2], (long long)n, f32 ? 1 : 0, (f32 && P == 0) ? 1 : 0, cf ? 1 : 0};
+  cudaError_t e = launch("block_sort", n, s, [&] { return var.block_sort(sa, tiles, s); });
+  if (e != cudaSuccess) return cuda_fail(e);
+  for (int i = 1; i <= P; ++i) {
+    const int src = (P - i + 1) % 2, dst = (P - i) % 2;
+    MergeArgs ma{bk[src], bv[src], bk[dst], bv[dst], (long long)n, T << (i - 1),
+                 (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0};
+    e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
+    if (e != cudaSuccess) return cuda_fail(e);
+  }
+  return BCF_SUCCESS;
+}
+
+// ---------------------------------------------------------------------------
+// distributed helpers
+// ---------------------------------------------------------------------------
+__global__ void split_counts_kernel(const uint32_t* __restrict__ a, unsigned long long n,
+                                    const uint32_t* __restrict__ piv, int npiv,
+                                    unsigned long long* __restrict__ lt, unsigned long long* __restrict__ le) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= npiv) return;
+  const uint32_t v = piv[i];
+  unsigned long long lo = 0, hi = n;  // first index with a[idx] >= v
+  while (lo < hi) {
+    const unsigned long long mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1; else hi = mid;
+  }
+  lt[i] = lo;
+  hi = n;  // first index with a[idx] > v
+  while (lo < hi) {
+    const unsigned long long mid = (lo + hi) >> 1;
+    if (a[mid] <= v) lo = mid + 1; else hi = mid;
+  }
+  le[i] = lo;
+}
+
+}  // namespace bcf
+
+using namespace bcf;
+
+extern "C" {
+
+void bcf_default_params(bcf_params* p) {
+  if (!p) return;
+  p->items_per_thread = DEFAULT_E;
+  p->block_threads = DEFAULT_U;
+  p->algo = BCF_ALGO_CONFLICT_FREE;
+}
+
+bcf_status bcf_sort_u32(const uint32_t* d_in, uint32_t* d_out, uint64_t n, void* d_temp,
+                        size_t* temp_bytes, const bcf_params* p, void* stream) {
+  return sort_impl(d_in, d_out, nullptr, nullptr, n, d_temp, temp_bytes, p, (cudaStream_t)stream, false,
+                   false);
+}
+
+bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_temp, size_t* temp_bytes,
+                        const bcf_params* p, void* stream) {
+  return sort_impl((const uint32_t*)d_in, (uint32_t*)d_out, nullptr, nullptr, n, d_temp, temp_bytes, p,
+                   (cudaStream_t)stream, true, false);
+}
+
+bcf_status bcf_sort_pairs_u32(const uint32_t* d_keys_in, uint32_t* d_keys_out, const uint32_t* d_vals_in,
+                              uint32_t* d_vals_out, uint64_t n, void* d_temp, size_t* temp_bytes,
+                              const bcf_params* p, void* stream) {
+  return sort_impl(d_keys_in, d_keys_out, d_vals_in, d_vals_out, n, d_temp, temp_bytes, p,
+                   (cudaStream_t)stream, false, true);
+}
+
+bcf_status bcf_worst_case_u32_host(uint32_t* h_out, uint64_t n, int32_t E, int32_t u, uint64_t seed) {
+  if (n > 0 && !h_out) return BCF_ERROR_INVALID_VALUE;
+  if (E < 2 || E > 32 || u < 32 || u % 32 != 0) return BCF_ERROR_UNSUPPORTED;
+  try {
+    wc::generate(h_out, n, E, u, seed);
+  } catch (...) {
+    return BCF_ERROR_INVALID_VALUE;
+  }
+  return BCF_SUCCESS;
+}
+
+bcf_status bcf_worst_case_u32(uint32_t* d_out, uint64_t n, int32_t E, int32_t u, uint64_t seed,
+                              void* stream) {
+  if (n > 0 && !d_out) return BCF_ERROR_INVALID_VALUE;
+  if (E < 2 || E > 32 || u < 32 || u % 32 != 0) return BCF_ERROR_UNSUPPORTED;
+  if (n == 0) return BCF_SUCCESS;
+  uint32_t* h = nullptr;
+  cudaError_t e = cudaMallocHost(&h, n * sizeof(uint32_t));
+  if (e != cudaSuccess) return cuda_fail(e);
+  bcf_status st = bcf_worst_case_u32_host(h, n, E, u, seed);
+  if (st == BCF_SUCCESS) {
+    e = cudaMemcpyAsync(d_out, h, n * sizeof(uint32_t), cudaMemcpyHostToDevice, (cudaStream_t)stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize((cudaStream_t)stream);
+    if (e != cudaSuccess) st = cuda_fail(e);
+  }
+  cudaFreeHost(h);
+  return st;
+}
+
+bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint32_t* d_pivots, int32_t npiv,
+                                uint64_t* d_lt_counts, uint64_t* d_le_counts, void* stream) {
+  if (npiv < 0) return BCF_ERROR_INVALID_VALUE;
+  if (npiv == 0) return BCF_SUCCESS;
+  if ((n > 0 && !d_sorted) || !d_pivots || !d_lt_counts || !d_le_counts) return BCF_ERROR_INVALID_VALUE;
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaError_t e = launch("split_counts", (uint64_t)npiv, s, [&] {
+    split_counts_kernel<<<(npiv + 127) / 128, 128, 0, s>>>(d_sorted, (unsigned long long)n, d_pivots, npiv,
+                                                          (unsigned long long*)d_lt_counts,
+                                                          (unsigned long long*)d_le_counts);
+    return cudaGetLastError();
+  });
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
+bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals, const uint64_t* h_run_offsets,
+                              int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals, void* d_temp,
+                              size_t* temp_bytes, const bcf_params* pp, void* stream) {
+  // Pairwise merge tree over the runs in run order (run 2g is A, 2g+1 is B,
+  // ties to A = the lower run), table mode of the CF merge-pass kernel.
+  if (!temp_bytes || nruns < 0 || (nruns > 0 && !h_run_offsets)) return BCF_ERROR_INVALID_VALUE;
+  Params p;
+  bcf_status st = resolve(pp, p);
+  if (st != BCF_SUCCESS) return st;
+  if (p.algo != BCF_ALGO_CONFLICT_FREE) return BCF_ERROR_UNSUPPORTED;
+  const bool pairs = d_run_vals != nullptr;
+  const uint64_t n = nruns > 0 ? h_run_offsets[nruns] : 0;
+  for (int r = 0; r < nruns; ++r)
+    if (h_run_offsets[r + 1] < h_run_offsets[r] || h_run_offsets[0] != 0) return BCF_ERROR_INVALID_VALUE;
+  const size_t key_bytes = align_up((size_t)n * sizeof(uint32_t), 256);
+  const size_t table_bytes = align_up(sizeof(GroupDesc) * (size_t)(nruns / 2 + 1), 256);
+  const size_t need = 256 + key_bytes * (pairs ? 2 : 1) + table_bytes * 64;
+  if (d_temp == nullptr) {
+    *temp_bytes = need;
+    return BCF_SUCCESS;
+  }
+  if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
+  if (n == 0) return BCF_SUCCESS;
+  if (!d_runs || !d_out || (pairs && !d_out_vals)) return BCF_ERROR_INVALID_VALUE;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (nruns == 1) {
+    cudaError_t e = cudaMemcpyAsync(d_out, d_runs, n * 4, cudaMemcpyDeviceToDevice, s);
+    if (e == cudaSuccess && pairs) e = cudaMemcpyAsync(d_out_vals, d_run_vals, n * 4, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+  }
+  const Variant& var = launch_table().v[p.E][u_index(p.U)][0][pairs ? 1 : 0];
+  if (!var.merge) return BCF_ERROR_UNSUPPORTED;
+  const long long T = (long long)p.U * p.E;
+  char* tb = (char*)align_up((size_t)d_temp, 256);
+  uint32_t* tk = (uint32_t*)tb;
+  uint32_t* tv = pairs ? (uint32_t*)(tb + key_bytes) : nullptr;
+  GroupDesc* dtab = (GroupDesc*)(tb + key_bytes * (pairs ? 2 : 1));
+  int P = 0;
+  while ((1 << P) < nruns) ++P;
+  std::vector<uint64_t> off(h_run_offsets, h_run_offsets + nruns + 1);
+  uint32_t* bk[2] = {d_out, tk};
+  uint32_t* bv[2] = {d_out_vals, tv};
+  const uint32_t* srck = d_runs;
+  const uint32_t* srcv = d_run_vals;
+  for (int i = 1; i <= P; ++i) {
+    const int dst = (P - i) % 2;
+    std::vector<GroupDesc> tab;
+    std::vector<uint64_t> noff{0};
+    long long tiles = 0;
+    const int nr = (int)off.size() - 1;
+    for (int r = 0; r < nr; r += 2) {
+      GroupDesc g{};
+      g.a_off = (long long)off[r];
+      g.na = (long long)(off[r + 1] - off[r]);
+      g.b_off = (long long)off[std::min(r + 1, nr)];
+      g.nb = r + 1 < nr ? (long long)(off[r + 2] - off[r + 1]) : 0;
+      g.out_off = g.a_off;
+      g.tile_begin = tiles;
+      tiles += (g.na + g.nb + T - 1) / T;
+      noff.push_back(off[std::min(r + 2, nr)]);
+      if (g.na + g.nb > 0) tab.push_back(g);
+    }
+    GroupDesc* dt = dtab + (size_t)(i - 1) * (table_bytes / sizeof(GroupDesc));
+    cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(e);
+    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, dt, (int)tab.size()};
+    e = launch("merge_runs", n, s, [&] { return var.merge(ma, tiles, s); });
+    if (e != cudaSuccess) return cuda_fail(e);
+    srck = bk[dst];
+    srcv = bv[dst];
+    off.swap(noff);
+  }
+  return BCF_SUCCESS;
+}
+
+const char* bcf_status_string(bcf_status s) {
+  switch (s) {
+    case BCF_SUCCESS: return "BCF_SUCCESS";
+    case BCF_ERROR_INVALID_VALUE: return "BCF_ERROR_INVALID_VALUE";
+    case BCF_ERROR_UNSUPPORTED: return "BCF_ERROR_UNSUPPORTED";
+    case BCF_ERROR_CUDA: return "BCF_ERROR_CUDA";
+    case BCF_ERROR_TEMP_TOO_SMALL: return "BCF_ERROR_TEMP_TOO_SMALL";
+  }
+  return "BCF_ERROR_UNKNOWN";
+}
+
+int32_t bcf_abi_version(void) { return BCF_ABI_VERSION; }
+int32_t bcf_last_cuda_error(void) { return t_last_cuda_error; }
+
+bcf_status bcf_profile_enable(int32_t on) {
+  g_prof_on.store(on ? 1 : 0);
+  return BCF_SUCCESS;
+}
+
+bcf_status bcf_profile_collect(bcf_kernel_stats* out, int32_t max, int32_t* count) {
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  std::vector<bcf_kernel_stats> acc;
+  cudaError_t err = cudaSuccess;
+  for (auto& r : g_recs) {
+    float ms = 0.f;
+    cudaError_t e = cudaEventSynchronize(r.b);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.a, r.b);
+    if (e != cudaSuccess) err = e;
+    auto it = std::find_if(acc.begin(), acc.end(), [&](const bcf_kernel_stats& k) { return std::strcmp(k.name, r.name) == 0; });
+    if (it == acc.end()) {
+      bcf_kernel_stats k{};
+      std::strncpy(k.name, r.name, sizeof(k.name) - 1);
+      acc.push_back(k);
+      it = acc.end() - 1;
+    }
+    it->launches += 1;
+    it->total_ms += ms;
+    it->keys += r.keys;
+    g_pool.push_back(r.a);
+    g_pool.push_back(r.b);
+  }
+  g_recs.clear();
+  if (count) *count = (int32_t)acc.size();
+  for (int i = 0; i < (int)acc.size() && i < max && out; ++i) out[i] = acc[i];
+  return err == cudaSuccess ? BCF_SUCCESS : cuda_fail(err);
+}
+
+int64_t bcf_launch_count(void) { return g_launches.load(); }
+
+}  // extern "C"

@@ -1,0 +1,470 @@
+// bcf_device.cuh -- device primitives of the bank-conflict-free (CF) mergesort.
+//
+// Notation follows Berney & Sitchinava, "Eliminating Bank Conflicts in GPU
+// Mergesort", SPAA'25: w = 32 banks / warp lanes, E items per
+// thread, d = GCD(w, E), u = U threads per block, tile T = U*E.
+//
+// Shared-memory tile layout (Alg. 1 line 2; §3.3):
+//     logical index k:  A[x] at k = x,  B[y] at k = T-1-y  (pi: B reversed)
+//     physical index  = rho(k): partitions of P = wE/d elements rotated right
+//                       by (partition mod d)            (§3.2)
+// With this layout every shared-memory instruction below touches, per warp,
+// a "round set" {k = j (mod E)} of one window of wE logical indices (or
+// consecutive physical words), which is a complete residue system mod w
+// (Lemma 1 / Corollary 3) -> zero bank conflicts for every input.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace bcf {
+
+constexpr int W = 32;  // banks = warp width on sm_100a (32 banks x 4 B)
+constexpr unsigned FULL = 0xffffffffu;
+
+__host__ __device__ constexpr int cgcd(int a, int b) { return b == 0 ? a : cgcd(b, a % b); }
+__host__ __device__ constexpr int clog2(int x) { return x <= 1 ? 0 : 1 + clog2(x >> 1); }
+__host__ __device__ constexpr int cpow2ceil(int x) { return x <= 1 ? 1 : 2 * cpow2ceil((x + 1) >> 1); }
+__host__ __device__ constexpr bool is_pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
+
+// ---------------------------------------------------------------------------
+// rho: logical -> physical shared-memory word.
+// Periodic with period wE (d partitions), so banks depend on k mod wE only.
+// ---------------------------------------------------------------------------
+template <int E>
+__device__ __forceinline__ int rho(int k) {
+  constexpr int d = cgcd(W, E);
+  if constexpr (d == 1) {
+    return k;
+  } else {
+    constexpr int P = W * E / d;
+    const int l = k / P;           // constant divisor
+    const int x = k - l * P;
+    int y = x + (l % d);
+    if (y >= P) y -= P;
+    return l * P + y;
+  }
+}
+
+template <int E>
+__device__ __forceinline__ int rho_inv(int p) {
+  constexpr int d = cgcd(W, E);
+  if constexpr (d == 1) {
+    return p;
+  } else {
+    constexpr int P = W * E / d;
+    const int l = p / P;
+    const int y = p - l * P;
+    int x = y - (l % d);
+    if (x < 0) x += P;
+    return l * P + x;
+  }
+}
+
+// First logical index of the next rho-partition after k (for splitting a run
+// of consecutive probes at the partition wrap).
+template <int E>
+__device__ __forceinline__ int rho_partition_end(int k) {
+  constexpr int d = cgcd(W, E);
+  constexpr int P = W * E / d;
+  return (k / P + 1) * P;
+}
+
+// ---------------------------------------------------------------------------
+// Run views in global memory.  A sorted run of `len` keys is stored either
+// ascending or descending (the CF pipeline stores every odd run of a pass
+// descending, so that the tile stage writes B reversed = pi(B) with unit-stride
+// reads).
+// ---------------------------------------------------------------------------
+struct RunView {
+  const uint32_t* base;
+  long long len;
+  int desc;  // 1: element y lives at base[len-1-y]
+  __device__ __forceinline__ long long addr(long long y) const { return desc ? (len - 1 - y) : y; }
+  __device__ __forceinline__ uint32_t ld(long long y) const { return __ldg(base + addr(y)); }
+};
+
+// ---------------------------------------------------------------------------
+// Merge path (Green et al. [24]): number of A elements among the
+// first D outputs of the stable merge of A and B (ties to A).  Warp-cooperative
+// 32-ary search over global memory: each round every lane tests one candidate
+// (2 independent loads), a ballot keeps the monotone prefix.  Returns the same
+// value to all lanes.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ long long merge_path_warp_global(const RunView& A, const RunView& B,
+                                                            long long D, int lane) {
+  long long lo = D - B.len;
+  if (lo < 0) lo = 0;
+  long long hi = D < A.len ? D : A.len;
+  // invariant: answer in [lo, hi]; Q(m) := a(D) >= m+1 := !(B[D-1-m] < A[m])
+  while (hi > lo) {
+    const long long cnt = hi - lo;
+    const long long s = (cnt + 31) >> 5;  // probe stride
+    const long long m = lo + (long long)(lane + 1) * s - 1;
+    bool p = false;
+    if (m < hi) {
+      const uint32_t a = A.ld(m);
+      const uint32_t b = B.ld(D - 1 - m);
+      p = !(b < a);
+    }
+    const int c = __popc(__ballot_sync(FULL, p));
+    const long long nlo = lo + (long long)c * s;
+    long long nhi = lo + (long long)(c + 1) * s - 1;
+    if (nhi > hi) nhi = hi;
+    lo = nlo;
+    hi = nhi;
+    if (s == 1) break;  // every candidate was tested: lo == answer
+  }
+  return lo;
+}
+
+// ---------------------------------------------------------------------------
+// Conflict-free warp-origin search in shared memory.
+// Returns a(D) for the merge group in smem (A[x] at logical base+x, B[y] at
+// base+S2-1-y, S2 = group size, a multiple of wE).
+// Probe stride s = fE with f odd: the 32 probes of a round are a round set of
+// a window (mod wE), hence conflict-free under rho.  The last <= E consecutive
+// probes are split at the rho-partition wrap.
+// ---------------------------------------------------------------------------
+template <int E>
+__device__ __forceinline__ int warp_origin_smem(const uint32_t* __restrict__ sk, int base, int S2,
+                                                int NA, int NB, int D, int lane) {
+  if (D > NA + NB) D = NA + NB;  // a(D) = NA past the end (ragged tile)
+  // A[x] at logical base+x; B[y] at base+S2-1-y, so B[D-1-m] at base+S2-D+m
+  const int bofs = base + S2 - D;
+  int lo = D - NB;
+  if (lo < 0) lo = 0;
+  int hi = D < NA ? D : NA;
+  while (hi - lo > E) {
+    const int cnt = hi - lo;
+    // stride s = f*E with f odd and 32*s >= cnt: the 32 probes are = const
+    // (mod E) and pairwise distinct mod wE -> a round set of a window.
+    const int need = (cnt + 31) >> 5;
+    int f = (need + E - 1) / E;
+    f |= 1;
+    const int s = f * E;
+    const int m = lo + (lane + 1) * s - 1;
+    bool p = false;
+    if (m < hi) {
+      const uint32_t a = sk[rho<E>(base + m)];
+      const uint32_t b = sk[rho<E>(bofs + m)];
+      p = !(b < a);
+    }
+    const int c = __popc(__ballot_sync(FULL, p));
+    const int nlo = lo + c * s;
+    int nhi = lo + (c + 1) * s - 1;
+    if (nhi > hi) nhi = hi;
+    lo = nlo;
+    hi = nhi;
+  }
+  // final: candidates m = lo + lane, lane < hi - lo (<= E)
+  const int m = lo + lane;
+  const bool act = m < hi;
+  uint32_t a = 0, b = 0;
+  constexpr int d = cgcd(W, E);
+  if constexpr (d == 1) {
+    if (act) {
+      a = sk[base + m];
+      b = sk[bofs + m];
+    }
+  } else {
+    const int aend = rho_partition_end<E>(base + lo);
+    const int bend = rho_partition_end<E>(bofs + lo);
+    if (act && base + m < aend) a = sk[rho<E>(base + m)];
+    __syncwarp();
+    if (act && base + m >= aend) a = sk[rho<E>(base + m)];
+    __syncwarp();
+    if (act && bofs + m < bend) b = sk[rho<E>(bofs + m)];
+    __syncwarp();
+    if (act && bofs + m >= bend) b = sk[rho<E>(bofs + m)];
+  }
+  const bool p = act && !(b < a);
+  return lo + __popc(__ballot_sync(FULL, p));
+}
+
+// ---------------------------------------------------------------------------
+// Conflict-free per-lane split search.
+// The lanes [wb, wb+WL) of a warp form one "window": their diagonals are
+// Dw + l'E (l' = lane - wb), the window's merge-path origin is alpha (so
+// beta = Dw - alpha).  A[x] at logical base+x, B[y] at logical base+S2-1-y
+// where S2 is the size of the merge group's tile/group (multiple of wE).
+// Returns a(Dw + l'E) for the calling lane.
+//   (2) corners: lane l' holds A[alpha+(l'+1)E-1] and B[beta+l'E] (stride E);
+//       coarse cell M = max{m <= l' : Q(alpha+mE)} by shuffle bisection;
+//   (3) cell scan: round j reads A[alpha+ME+j] and B[beta+(l'-M)E-1-j].
+// ---------------------------------------------------------------------------
+template <int E>
+__device__ __forceinline__ int lane_split_smem(const uint32_t* __restrict__ sk, int base, int S2,
+                                               int NA, int NB, int Dw, int alpha, int lane, int WL) {
+  const int wb = lane & ~(WL - 1);
+  const int lp = lane - wb;
+  const int beta = Dw - alpha;
+  const int D = Dw + lp * E;
+  // corners
+  const int ia = alpha + (lp + 1) * E - 1;
+  const int ib = beta + lp * E;
+  uint32_t cA = 0, cB = 0;
+  if (ia < NA) cA = sk[rho<E>(base + ia)];
+  if (ib < NB) cB = sk[rho<E>(base + S2 - 1 - ib)];
+  // coarse: largest m in [0, lp] with Q(alpha + mE)
+  int lo = 0, hi = lp + 1;  // Q(lo) true, answer < hi
+#pragma unroll
+  for (int it = 0; it < 6; ++it) {  // ceil(log2(33)) bisection steps
+    const int mid = (lo + hi) >> 1;
+    const int m = (hi - lo > 1) ? mid : lo;
+    const int srcA = wb + (m >= 1 ? m - 1 : 0);
+    const int srcB = wb + (lp - m >= 0 ? lp - m : 0);
+    const uint32_t a = __shfl_sync(FULL, cA, srcA);
+    const uint32_t b = __shfl_sync(FULL, cB, srcB);
+    if (hi - lo > 1) {
+      const bool validA = alpha + m * E <= NA;
+      const bool validB = beta + (lp - m) * E < NB;
+      const bool q = (m == 0) || (validA && (!validB || !(b < a)));
+      if (q) lo = m; else hi = m;
+    }
+  }
+  const int ac = alpha + lo * E;  // a(D) in [ac, ac+E]
+  int cnt = 0;
+#pragma unroll
+  for (int j = 0; j < E; ++j) {
+    const int a = ac + j + 1;  // candidate a(D) >= a ?
+    const bool inA = a <= NA && a <= D;
+    const bool needB = (D - a) < NB;
+    uint32_t ka = 0, kb = 0;
+    if (inA) ka = sk[rho<E>(base + a - 1)];
+    if (inA && needB) kb = sk[rho<E>(base + S2 - 1 - (D - a))];
+    const bool q = inA && (!needB || !(kb < ka));
+    cnt += q ? 1 : 0;
+  }
+  return ac + cnt;
+}
+
+// ---------------------------------------------------------------------------
+// Alg. 1 DUAL-SUBSEQUENCE-GATHER.  Thread with A offset a,
+// B offset b (in its merge group), |A_i| = nA, |B_i| = nB (nA+nB <= E; fewer
+// only in a ragged tile: those rounds read nothing and hold a pad).
+// k = a mod E; round j reads A_i[(j-k) mod E] if that index < nA, else
+// B_i[(k-j-1) mod E]; both at logical base + idx, B reversed behind A.
+// After the gather, items[] is a circular bitonic sequence starting at k.
+// ---------------------------------------------------------------------------
+template <int E, bool PAIRS>
+__device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restrict__ sk,
+                                                        const uint32_t* __restrict__ sv, int base,
+                                                        int S2, int a, int b, int nA, int nB,
+                                                        uint32_t (&key)[E], uint32_t (&val)[E],
+                                                        uint32_t pad) {
+  const int k = a % E;
+  const int baseA = base + a;
+  const int baseB = base + S2 - b - E;  // B_i[E-1-ia] at base+S2-1-(b+E-1-ia) = baseB+ia
+#pragma unroll
+  for (int j = 0; j < E; ++j) {
+    int ia = j - k;
+    if (ia < 0) ia += E;
+    const bool isA = ia < nA;
+    const bool ok = isA || (E - 1 - ia) < nB;
+    const int idx = rho<E>((isA ? baseA : baseB) + ia);
+    if (ok) {
+      key[j] = sk[idx];
+      if constexpr (PAIRS) val[j] = sv[idx];
+    } else {
+      key[j] = pad;
+      if constexpr (PAIRS) val[j] = 0;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Compare-exchange helpers.  Keys-only: plain min/max (equal keys are equal
+// bit patterns, so order among them is unobservable).  Pairs: lexicographic
+// (key, tag) where tag is the element's rank in the stable order of the two
+// inputs -- a strict total order, so any sorting network yields the stable
+// result.
+// ---------------------------------------------------------------------------
+template <bool PAIRS>
+struct Elem;
+
+template <>
+struct Elem<false> {
+  __device__ __forceinline__ static void ce(uint32_t& k0, uint32_t& k1, uint32_t&, uint32_t&,
+                                            uint32_t&, uint32_t&) {
+    const uint32_t lo = min(k0, k1);
+    const uint32_t hi = max(k0, k1);
+    k0 = lo;
+    k1 = hi;
+  }
+};
+
+template <>
+struct Elem<true> {
+  __device__ __forceinline__ static void ce(uint32_t& k0, uint32_t& k1, uint32_t& t0, uint32_t& t1,
+                                            uint32_t& v0, uint32_t& v1) {
+    const bool sw = (k1 < k0) || (k1 == k0 && t1 < t0);
+    const uint32_t nk0 = sw ? k1 : k0, nk1 = sw ? k0 : k1;
+    const uint32_t nt0 = sw ? t1 : t0, nt1 = sw ? t0 : t1;
+    const uint32_t nv0 = sw ? v1 : v0, nv1 = sw ? v0 : v1;
+    k0 = nk0; k1 = nk1; t0 = nt0; t1 = nt1; v0 = nv0; v1 = nv1;
+  }
+};
+
+// Virtual-pad bookkeeping for networks padded from E to N = 2^ceil(log2 E):
+// positions [E, N) hold virtual keys (-inf for the merger, +inf for the sort)
+// whose comparisons resolve at compile time into moves.
+template <int N>
+struct PadMask {
+  __host__ __device__ static constexpr unsigned all() { return N >= 32 ? 0xffffffffu : ((1u << N) - 1u); }
+};
+
+// Bitonic merger (Batcher) ascending over N = 2^ceil(log2 E) slots; slots
+// [E, N) are virtual -inf.  Input must be bitonic (up-then-down, cyclically).
+template <int E, bool PAIRS>
+__device__ __forceinline__ void bitonic_merge_pad(uint32_t (&k)[E], uint32_t (&t)[E], uint32_t (&v)[E]) {
+  constexpr int N = cpow2ceil(E);
+  constexpr int LOGN = clog2(N);
+  uint32_t K[N], Tg[N], V[N];
+#pragma unroll
+  for (int i = 0; i < N; ++i) {
+    K[i] = i < E ? k[i] : 0u;
+    if constexpr (PAIRS) { Tg[i] = i < E ? t[i] : 0u; V[i] = i < E ? v[i] : 0u; }
+  }
+  unsigned virt = PadMask<N>::all() & ~((E >= 32) ? 0xffffffffu : ((1u << E) - 1u));
+#pragma unroll
+  for (int ls = LOGN - 1; ls >= 0; --ls) {
+    const int s = 1 << ls;
+    unsigned nvirt = virt;
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      if ((i & s) == 0) {
+        const int j = i + s;
+        const bool vi = (virt >> i) & 1u, vj = (virt >> j) & 1u;
+        if (!vi && !vj) {
+          Elem<PAIRS>::ce(K[i], K[j], Tg[i], Tg[j], V[i], V[j]);
+        } else if (!vi && vj) {
+          // min(-inf, x) = -inf goes to i, x moves to j
+          K[j] = K[i];
+          if constexpr (PAIRS) { Tg[j] = Tg[i]; V[j] = V[i]; }
+          nvirt = (nvirt | (1u << i)) & ~(1u << j);
+        }
+      }
+    }
+    virt = nvirt;
+  }
+  // the N-E virtual -inf ended at slots [0, N-E): real outputs are [N-E, N)
+#pragma unroll
+  for (int i = 0; i < E; ++i) {
+    k[i] = K[N - E + i];
+    if constexpr (PAIRS) { t[i] = Tg[N - E + i]; v[i] = V[N - E + i]; }
+  }
+}
+
+// Batcher odd-even merge sort ascending over N = 2^ceil(log2 E) slots; slots
+// [E, N) are virtual +inf.  Used for the per-thread sort of E keys in the block
+// sort (the paper uses Thrust's odd-even transposition sort; any
+// network producing the same result is acceptable, reading c15).
+template <int E, bool PAIRS>
+__device__ __forceinline__ void oddeven_sort_pad(uint32_t (&k)[E], uint32_t (&t)[E], uint32_t (&v)[E]) {
+  constexpr int N = cpow2ceil(E);
+  constexpr int LOGN = clog2(N);
+  uint32_t K[N], Tg[N], V[N];
+#pragma unroll
+  for (int i = 0; i < N; ++i) {
+    K[i] = i < E ? k[i] : 0u;
+    if constexpr (PAIRS) { Tg[i] = i < E ? t[i] : 0u; V[i] = i < E ? v[i] : 0u; }
+  }
+  unsigned virt = PadMask<N>::all() & ~((E >= 32) ? 0xffffffffu : ((1u << E) - 1u));
+#pragma unroll
+  for (int lp = 0; lp < LOGN; ++lp) {
+    const int p = 1 << lp;
+#pragma unroll
+    for (int lk = lp; lk >= 0; --lk) {
+      const int kk = 1 << lk;
+      const int j0 = (kk == p) ? 0 : kk;  // kk % p
+      unsigned nvirt = virt;
+#pragma unroll
+      for (int x = 0; x < N; ++x) {
+        const int y = x + kk;
+        if (x >= j0 && ((x - j0) % (2 * kk)) < kk && y < N && (x / (2 * p)) == (y / (2 * p))) {
+          const bool vx = (virt >> x) & 1u, vy = (virt >> y) & 1u;
+          if (!vx && !vy) {
+            Elem<PAIRS>::ce(K[x], K[y], Tg[x], Tg[y], V[x], V[y]);
+          } else if (vx && !vy) {
+            // max(+inf, y) = +inf goes to y, y's value moves to x
+            K[x] = K[y];
+            if constexpr (PAIRS) { Tg[x] = Tg[y]; V[x] = V[y]; }
+            nvirt = (nvirt | (1u << y)) & ~(1u << x);
+          }
+        }
+      }
+      virt = nvirt;
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < E; ++i) {
+    k[i] = K[i];
+    if constexpr (PAIRS) { t[i] = Tg[i]; v[i] = V[i]; }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// In-register merge of the gathered registers (PAPER.md:354 uses Thrust's
+// odd-even transposition sort; reading c15 allows any data-oblivious network
+// with the same result).  items[] holds, circularly from k = a mod E,
+// A_i ascending then B_i descending (bitonic).
+//   E = 2^x: the bitonic merger sorts any cyclic shift directly.
+//   otherwise: barrel-rotate left by k (static stages), pad with -inf, merge.
+// Pairs: tag = rank in the stable order of A_i ++ B_i (pads: E).
+// ---------------------------------------------------------------------------
+template <int E, bool PAIRS>
+__device__ __forceinline__ void merge_registers(uint32_t (&key)[E], uint32_t (&val)[E], int a, int nA,
+                                                int nB) {
+  const int k = a % E;
+  uint32_t tag[E];
+  if constexpr (is_pow2(E)) {
+    if constexpr (PAIRS) {
+#pragma unroll
+      for (int j = 0; j < E; ++j) {
+        int ia = j - k;
+        if (ia < 0) ia += E;
+        const int ib = E - 1 - ia;
+        tag[j] = ia < nA ? (uint32_t)ia : (ib < nB ? (uint32_t)(nA + ib) : (uint32_t)E);
+      }
+    }
+    bitonic_merge_pad<E, PAIRS>(key, tag, val);
+  } else {
+    // rotate left by k: new[m] = old[(m + k) mod E]
+    constexpr int NBITS = clog2(E - 1) + 1;  // bits of k in [0, E-1]
+#pragma unroll
+    for (int bit = 0; bit < NBITS; ++bit) {
+      const int sh = 1 << bit;
+      if ((k >> bit) & 1) {
+        uint32_t tk[E], tv[E];
+#pragma unroll
+        for (int m = 0; m < E; ++m) {
+          tk[m] = key[(m + sh) % E];
+          if constexpr (PAIRS) tv[m] = val[(m + sh) % E];
+        }
+#pragma unroll
+        for (int m = 0; m < E; ++m) {
+          key[m] = tk[m];
+          if constexpr (PAIRS) val[m] = tv[m];
+        }
+      }
+    }
+    if constexpr (PAIRS) {
+#pragma unroll
+      for (int m = 0; m < E; ++m) {
+        const int ib = E - 1 - m;
+        tag[m] = m < nA ? (uint32_t)m : (ib < nB ? (uint32_t)(nA + ib) : (uint32_t)E);
+      }
+    }
+    bitonic_merge_pad<E, PAIRS>(key, tag, val);
+  }
+}
+
+// f32 <-> order-preserving u32 (IEEE totalOrder, reading c2)
+__device__ __forceinline__ uint32_t f32_encode(uint32_t b) {
+  return b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u);
+}
+__device__ __forceinline__ uint32_t f32_decode(uint32_t u) {
+  return u ^ ((~(uint32_t)((int32_t)u >> 31)) | 0x80000000u);
+}
+
+}  // namespace bcf

@@ -1,0 +1,398 @@
+// bcf_kernels.cuh -- the three hot-path kernels of the pairwise mergesort
+// (PAPER.md:59-61, :348-354), each in two variants:
+//   CF       the paper's bank-conflict-free design (pi + rho layout, Alg. 1
+//            gather, conflict-free split search, in-register merge network);
+//   BASELINE the unmodified Thrust design the paper measures against
+//            (A|B forward in shared memory, per-thread binary merge path,
+//            serial merge reading shared memory) -- keys only.
+//
+// block_sort  one CTA sorts a tile of T = U*E keys: per-thread sort of E keys,
+//             then log2(U) merge levels in shared memory.
+// merge_pass  one CTA produces one output tile of T keys of a pairwise merge
+//             of runs of R keys (merge-path tile split fused in).
+//
+// Global run directions (CF only): in every pass run r is stored descending
+// iff r is odd, so a tile's B range, read with unit stride, lands in shared
+// memory already reversed (pi).  The final run (index 0) is
+// ascending.  The baseline keeps every run ascending.
+#pragma once
+#include "bcf_device.cuh"
+
+namespace bcf {
+
+constexpr uint32_t PAD_KEY = 0xffffffffu;
+
+// dynamic shared memory of one CTA
+template <int E, int U, bool PAIRS>
+constexpr size_t tile_smem_bytes() {
+  return (size_t)(U * E + 1) * sizeof(uint32_t) * (PAIRS ? 2 : 1);
+}
+
+struct SortArgs {
+  const uint32_t* in_k;
+  const uint32_t* in_v;
+  uint32_t* out_k;
+  uint32_t* out_v;
+  long long n;
+  int encode_f32;  // encode f32 -> totalOrder u32 on load (block sort)
+  int decode_f32;  // decode on the final store
+  int cf_dirs;     // CF run directions (odd runs descending)
+};
+
+// One merge group: A = src[a_off, a_off+na), B = src[b_off, b_off+nb),
+// output dst[out_off, out_off+na+nb); *_desc: run stored descending.
+struct GroupDesc {
+  long long a_off, na, b_off, nb, out_off, tile_begin;
+  int a_desc, b_desc, out_desc, pad_;
+};
+
+struct MergeArgs {
+  const uint32_t* src_k;
+  const uint32_t* src_v;
+  uint32_t* dst_k;
+  uint32_t* dst_v;
+  long long n;
+  long long R;     // input run length (regular mode)
+  int decode_f32;  // final pass of an f32 sort
+  int cf_dirs;     // regular mode: odd runs descending
+  const GroupDesc* groups;  // table mode (merge of arbitrary runs) if non-null
+  int ngroups;
+};
+
+// Group of output tile `tile`: regular pairwise pass (run 2g with run 2g+1,
+// run r descending iff r odd under CF directions) or an explicit table.
+__device__ __forceinline__ GroupDesc group_of_tile(const MergeArgs& args, long long tile, int T,
+                                                   long long& j) {
+  GroupDesc G;
+  if (args.groups == nullptr) {
+    const long long tpg = (2 * args.R) / T;  // tiles per full group
+    const long long g = tile / tpg;
+    j = tile - g * tpg;
+    const long long g0 = g * 2 * args.R;
+    const long long left = args.n - g0;
+    G.a_off = g0;
+    G.na = left < args.R ? left : args.R;
+    G.b_off = g0 + args.R;
+    G.nb = left - G.na < args.R ? left - G.na : args.R;
+    G.out_off = g0;
+    G.tile_begin = g * tpg;
+    G.a_desc = 0;
+    G.b_desc = args.cf_dirs;
+    G.out_desc = args.cf_dirs && (g & 1);
+  } else {
+    int lo = 0, hi = args.ngroups - 1;  // last group with tile_begin <= tile
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (args.groups[mid].tile_begin <= tile) lo = mid; else hi = mid - 1;
+    }
+    G = args.groups[lo];
+    j = tile - G.tile_begin;
+  }
+  return G;
+}
+
+// ---------------------------------------------------------------------------
+// Output stage shared by both kernels: registers -> shared (round sets, rho
+// layout) -> coalesced global stores.  Thread's items are tile outputs
+// [D, D+E); `desc` writes the tile mirrored into a descending run whose
+// global element o lives at c0 + (T-1-o) ... expressed as gaddr = c0 + q with
+// q the logical smem index.
+// ---------------------------------------------------------------------------
+template <int E, int U, bool PAIRS>
+__device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uint32_t (&key)[E],
+                                           const uint32_t (&val)[E], int D, int cnt, bool desc,
+                                           uint32_t* __restrict__ gk, uint32_t* __restrict__ gv,
+                                           long long c0, bool decode) {
+  constexpr int T = U * E;
+  // round m: ascending -> item m at D+m; descending -> item E-1-m at T-E-D+m
+  const int base = desc ? (T - E - D) : D;
+#pragma unroll
+  for (int m = 0; m < E; ++m) {
+    const int idx = rho<E>(base + m);
+    sk[idx] = desc ? key[E - 1 - m] : key[m];
+    if constexpr (PAIRS) sv[idx] = desc ? val[E - 1 - m] : val[m];
+  }
+  __syncthreads();
+  const int qlo = desc ? T - cnt : 0;
+  const int qhi = desc ? T : cnt;
+#pragma unroll
+  for (int r = 0; r < E; ++r) {
+    const int P = threadIdx.x + r * U;  // physical word: consecutive per warp
+    const int q = rho_inv<E>(P);
+    if (q >= qlo && q < qhi) {
+      uint32_t x = sk[P];
+      if (decode) x = f32_decode(x);
+      gk[c0 + q] = x;
+      if constexpr (PAIRS) gv[c0 + q] = sv[P];
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Block sort (K1): tile t of T = U*E input keys -> sorted run t (descending
+// iff t odd under CF directions).
+// ---------------------------------------------------------------------------
+template <int E, int U, bool PAIRS, bool CF>
+__global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
+  constexpr int T = U * E;
+  constexpr int NW = U / W;
+  extern __shared__ uint32_t smem_dyn[];
+  uint32_t* sk = smem_dyn;                 // T + 1 keys
+  uint32_t* sv = smem_dyn + (T + 1);       // T + 1 values (pairs only)
+  __shared__ int s_org[NW + 1];
+  const int tid = threadIdx.x;
+  const int lane = tid & (W - 1);
+  const int warp = tid >> 5;
+  const long long tile = blockIdx.x;
+  const long long t0 = tile * T;
+  const long long rem = args.n - t0;
+  const int cnt = rem < T ? (int)rem : T;
+
+  // --- load: coalesced in physical order, pads = max key (they sort last and
+  // are trimmed by the count; stable order keeps them after real max keys).
+  {
+    uint32_t vk[E], vv[E];
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+      const int P = tid + r * U;
+      const int p = CF ? rho_inv<E>(P) : P;
+      vk[r] = PAD_KEY;
+      vv[r] = 0;
+      if (p < cnt) {
+        uint32_t x = __ldg(args.in_k + t0 + p);
+        if (args.encode_f32) x = f32_encode(x);
+        vk[r] = x;
+        if constexpr (PAIRS) vv[r] = __ldg(args.in_v + t0 + p);
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+      sk[tid + r * U] = vk[r];
+      if constexpr (PAIRS) sv[tid + r * U] = vv[r];
+    }
+  }
+  __syncthreads();
+  uint32_t key[E], val[E], tag[E];
+  // blocked read: round m reads logical tid*E + m (a round set)
+#pragma unroll
+  for (int m = 0; m < E; ++m) {
+    const int idx = CF ? rho<E>(tid * E + m) : tid * E + m;
+    key[m] = sk[idx];
+    if constexpr (PAIRS) { val[m] = sv[idx]; tag[m] = m; }
+  }
+  oddeven_sort_pad<E, PAIRS>(key, tag, val);
+
+  // --- log2(U) merge levels: runs of S = E*2^l, groups of G = 2^(l+1) threads
+#pragma unroll 1
+  for (int l = 0; (1 << l) < U; ++l) {
+    const int S = E << l;
+    const int G = 2 << l;
+    const int ir = tid & ((1 << l) - 1);   // index within its run
+    const int run = tid >> l;
+    const int gbase = (run >> 1) * 2 * S;  // group base (logical)
+    const bool isB = run & 1;
+    __syncthreads();
+    if constexpr (CF) {
+      // conflict-free scatter (fn. 5): B runs are written
+      // reversed (pi); in round m B-run lanes write item E-1-m so that every
+      // lane writes logical index = m (mod E).
+      const int base = isB ? gbase + 2 * S - E - ir * E : gbase + ir * E;
+#pragma unroll
+      for (int m = 0; m < E; ++m) {
+        const int idx = rho<E>(base + m);
+        sk[idx] = isB ? key[E - 1 - m] : key[m];
+        if constexpr (PAIRS) sv[idx] = isB ? val[E - 1 - m] : val[m];
+      }
+    } else {
+      const int base = gbase + (isB ? S : 0) + ir * E;
+#pragma unroll
+      for (int m = 0; m < E; ++m) sk[base + m] = key[m];
+    }
+    __syncthreads();
+    const int ig = tid & (G - 1);
+    const int D = ig * E;
+    if constexpr (CF) {
+      int alpha = 0, Dw = 0, WL = G;
+      if (G > W) {
+        Dw = (ig >> 5) * (W * E);
+        alpha = warp_origin_smem<E>(sk, gbase, 2 * S, S, S, Dw, lane);
+        WL = W;
+        if (lane == 0) s_org[warp] = alpha;
+      }
+      __syncthreads();
+      const int a = lane_split_smem<E>(sk, gbase, 2 * S, S, S, Dw, alpha, lane, WL);
+      int anext = __shfl_down_sync(FULL, a, 1);
+      if ((lane & (WL - 1)) == WL - 1) {
+        // last lane of the window: next window's origin, or the group end
+        anext = (G > W && ((ig >> 5) + 1) * W < G) ? s_org[warp + 1] : S;
+      }
+      const int nA = anext - a;
+      const int nB = E - nA;
+      const int b = D - a;
+      dual_subsequence_gather<E, PAIRS>(sk, sv, gbase, 2 * S, a, b, nA, nB, key, val, PAD_KEY);
+      merge_registers<E, PAIRS>(key, val, a, nA, nB);
+    } else {
+      // unmodified Thrust: per-thread binary merge path, then serial merge
+      // reading shared memory
+      const int abase = gbase, bbase = gbase + S;
+      int lo = D - S < 0 ? 0 : D - S;
+      int hi = D < S ? D : S;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (sk[bbase + D - 1 - mid] < sk[abase + mid]) hi = mid; else lo = mid + 1;
+      }
+      int ab = abase + lo, bb = bbase + (D - lo);
+      const int ae = abase + S, be = bbase + S;
+      uint32_t k1 = sk[ab], k2 = sk[bb];
+#pragma unroll
+      for (int m = 0; m < E; ++m) {
+        const bool p = (bb < be) && ((ab >= ae) || (k2 < k1));
+        key[m] = p ? k2 : k1;
+        if (p) ++bb; else ++ab;
+        const uint32_t x = sk[p ? bb : ab];
+        if (p) k2 = x; else k1 = x;
+      }
+    }
+  }
+  __syncthreads();
+  // --- store run `tile`: descending iff tile odd (CF directions)
+  const bool desc = args.cf_dirs && (tile & 1);
+  const long long c0 = desc ? t0 + cnt - T : t0;
+  store_tile<E, U, PAIRS>(sk, sv, key, val, tid * E, cnt, desc, args.out_k, args.out_v, c0,
+                          args.decode_f32 != 0);
+}
+
+// ---------------------------------------------------------------------------
+// Merge pass (K2+K3 fused): output tile `blockIdx.x` of the pairwise merge of
+// runs of R keys.  Group g merges run 2g (A) with run 2g+1 (B).
+// ---------------------------------------------------------------------------
+template <int E, int U, bool PAIRS, bool CF>
+__global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
+  constexpr int T = U * E;
+  constexpr int NW = U / W;
+  extern __shared__ uint32_t smem_dyn[];
+  uint32_t* sk = smem_dyn;                 // T + 1 keys
+  uint32_t* sv = smem_dyn + (T + 1);       // T + 1 values (pairs only)
+  __shared__ int s_org[NW + 1];
+  __shared__ long long s_split[2];
+  const int tid = threadIdx.x;
+  const int lane = tid & (W - 1);
+  const int warp = tid >> 5;
+  const long long tile = blockIdx.x;
+  long long j;
+  const GroupDesc grp = group_of_tile(args, tile, T, j);
+  const long long lenG = grp.na + grp.nb;
+  RunView Av{args.src_k + grp.a_off, grp.na, grp.a_desc};
+  RunView Bv{args.src_k + grp.b_off, grp.nb, grp.b_desc};
+  const long long D0 = j * T;
+  const long long D1 = D0 + T < lenG ? D0 + T : lenG;
+
+  // --- tile split by warp-cooperative merge path over global memory
+  if (warp < 2) {
+    const long long D = warp == 0 ? D0 : D1;
+    const long long a = merge_path_warp_global(Av, Bv, D, lane);
+    if (lane == 0) s_split[warp] = a;
+  }
+  __syncthreads();
+  const long long a0 = s_split[0];
+  const long long a1 = s_split[1];
+  const int cnt = (int)(D1 - D0);
+  const int NA = (int)(a1 - a0);
+  const int NB = cnt - NA;
+  const long long b0 = D0 - a0;
+
+  // --- staging: A forward at logical [0, NA); B reversed (CF: B[y] at T-1-y)
+  // or forward behind A (baseline).  Physical-order, coalesced global reads.
+  {
+    uint32_t vk[E], vv[E];
+    bool ok[E];
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+      const int P = tid + r * U;
+      ok[r] = false;
+      vk[r] = 0;
+      vv[r] = 0;
+      if constexpr (CF) {
+        const int q = rho_inv<E>(P);
+        if (q < NA) {
+          ok[r] = true;
+          const long long ga = Av.addr(a0 + q);
+          vk[r] = __ldg(Av.base + ga);
+          if constexpr (PAIRS) vv[r] = __ldg(args.src_v + grp.a_off + ga);
+        } else if (q >= T - NB) {
+          ok[r] = true;
+          const long long gb = Bv.addr(b0 + (T - 1 - q));
+          vk[r] = __ldg(Bv.base + gb);
+          if constexpr (PAIRS) vv[r] = __ldg(args.src_v + grp.b_off + gb);
+        }
+      } else {
+        if (P < NA) {
+          ok[r] = true;
+          vk[r] = __ldg(Av.base + Av.addr(a0 + P));
+        } else if (P < cnt) {
+          ok[r] = true;
+          vk[r] = __ldg(Bv.base + Bv.addr(b0 + (P - NA)));
+        }
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+      if (ok[r]) {
+        sk[tid + r * U] = vk[r];
+        if constexpr (PAIRS) sv[tid + r * U] = vv[r];
+      }
+    }
+  }
+  __syncthreads();
+
+  uint32_t key[E], val[E];
+  const int D = tid * E;
+  if constexpr (CF) {
+    const int Dw = warp * W * E;
+    const int alpha = warp_origin_smem<E>(sk, 0, T, NA, NB, Dw, lane);
+    if (lane == 0) s_org[warp] = alpha;
+    if (tid == 0) s_org[NW] = NA;
+    __syncthreads();
+    const int a = lane_split_smem<E>(sk, 0, T, NA, NB, Dw, alpha, lane, W);
+    int anext = __shfl_down_sync(FULL, a, 1);
+    if (lane == W - 1) anext = s_org[warp + 1];
+    const int Dc = D < cnt ? D : cnt;
+    const int Dn = D + E < cnt ? D + E : cnt;
+    const int nA = anext - a;
+    const int nB = (Dn - Dc) - nA;
+    const int b = Dc - a;
+    dual_subsequence_gather<E, PAIRS>(sk, sv, 0, T, a, b, nA, nB, key, val, PAD_KEY);
+    merge_registers<E, PAIRS>(key, val, a, nA, nB);
+  } else {
+    if (D < cnt) {
+      int lo = D - NB < 0 ? 0 : D - NB;
+      int hi = D < NA ? D : NA;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (sk[NA + D - 1 - mid] < sk[mid]) hi = mid; else lo = mid + 1;
+      }
+      int ab = lo, bb = NA + (D - lo);
+      const int ae = NA, be = NA + NB;
+      uint32_t k1 = sk[ab], k2 = sk[bb];
+#pragma unroll
+      for (int m = 0; m < E; ++m) {
+        const bool p = (bb < be) && ((ab >= ae) || (k2 < k1));
+        key[m] = p ? k2 : k1;
+        if (p) ++bb; else ++ab;
+        const uint32_t x = sk[p ? bb : ab];
+        if (p) k2 = x; else k1 = x;
+      }
+    } else {
+#pragma unroll
+      for (int m = 0; m < E; ++m) key[m] = PAD_KEY;
+    }
+  }
+  __syncthreads();
+  // --- output tile into the group's output run (descending if grp.out_desc)
+  const bool desc = grp.out_desc != 0;
+  const long long c0 = desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
+  store_tile<E, U, PAIRS>(sk, sv, key, val, D, cnt, desc, args.dst_k, args.dst_v, c0,
+                          args.decode_f32 != 0);
+}
+
+}  // namespace bcf
