@@ -1,0 +1,374 @@
+#!/usr/bin/env python
+"""bench.py -- headline benchmark of the B200 bank-conflict-free mergesort.
+
+Metric (BASELINE.json): sorted keys/s (32-bit) on uniform-random vs constructed
+worst-case inputs, their ratio, and (via ncu, profiles/) shared-memory bank
+conflicts.  Workload at N = 1: BASELINE.json configs[1], 2^24 uint32 keys,
+random vs worst-case, 1 x B200.  A step = one full sort (block sort + every
+merge pass) of one batch of 2^24 keys already resident in HBM; timed steps
+alternate random / worst-case (ABAB) so clock drift cancels in the ratio; L2
+is flushed (256 MiB write) between timed steps, outside the events.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+N > 1 (torchrun, one rank per GPU, NCCL): each rank holds 2^24 keys (weak
+scaling) and a step is the distributed sort (local sort, exact splitters,
+all_to_all, run merge).  Rank 0 prints ONE JSON line.
+`--impl reference` times the CPU oracle (plain stable mergesort, 1 core) on a
+bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synthetic_inputs as si  # noqa: E402
+
+METRIC = "sorted keys/s (32-bit) random vs worst-case, ratio; SMEM bank conflicts (ncu)"
+UNIT = "keys/s"
+WORKLOAD = "2^24 uint32 keys, random vs worst-case bank-conflict input, 1xB200 (BASELINE configs[1])"
+L2_FLUSH_BYTES = 256 << 20
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--log2n", type=int, default=24)
+    ap.add_argument("--E", type=int, default=0)
+    ap.add_argument("--u", type=int, default=0)
+    ap.add_argument("--algo", type=int, default=0)
+    ap.add_argument("--no-extras", action="store_true", help="skip e2e/cpu_baseline/contrast legs")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0}, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons during the timed region."""
+
+    REASONS = [
+        ("nvmlClocksEventReasonHwSlowdown", "hw_slowdown"),
+        ("nvmlClocksEventReasonHwThermalSlowdown", "hw_thermal_slowdown"),
+        ("nvmlClocksEventReasonSwThermalSlowdown", "sw_thermal_slowdown"),
+        ("nvmlClocksEventReasonSwPowerCap", "sw_power_cap"),
+        ("nvmlClocksEventReasonHwPowerBrakeSlowdown", "hw_power_brake_slowdown"),
+        ("nvmlClocksEventReasonApplicationsClocksSetting", "applications_clocks_setting"),
+        ("nvmlClocksEventReasonSyncBoost", "sync_boost"),
+    ]
+
+    def __init__(self, index: int):
+        self.ok = False
+        self.samples = []
+        self.reasons = set()
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:  # noqa: BLE001
+            self.max_mhz = None
+        self._stop = threading.Event()
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for attr, name in self.REASONS:
+                    if r & getattr(nv, attr, 0):
+                        self.reasons.add(name)
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def cpu_oracle_rate(n_sample: int, reps: int, kinds, E, u):
+    """The oracle (plain stable mergesort in C, 1 thread) on bounded samples."""
+    import oracle
+    from oracle import worstcase as wc
+
+    total_keys, total_s = 0, 0.0
+    for i in range(reps):
+        kind = kinds[i % len(kinds)]
+        if kind == "random":
+            x = si.uniform_u32(n_sample, si.config_seed(1) + i)
+        else:
+            x = wc.worst_case_input(n_sample, E, u, si.config_seed(1) + i)
+        t = time.perf_counter()
+        oracle.sort_u32(x)
+        total_s += time.perf_counter() - t
+        total_keys += n_sample
+    return total_keys / total_s, total_s
+
+
+def run_reference(a):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import paper_conf_spaa_berneys25_b200 as bcf  # only for the default (E, u) used by the worst case
+
+    try:
+        p = bcf.default_params()
+        E, u = a.E or p.items_per_thread, a.u or p.block_threads
+    except Exception:  # noqa: BLE001
+        E, u = a.E or 16, a.u or 256
+    n_full = 1 << a.log2n
+    n_sample = min(n_full, 1 << 21)
+    import oracle
+    from oracle import worstcase as wc
+
+    inputs = [si.uniform_u32(n_sample, si.config_seed(1)), wc.worst_case_input(n_sample, E, u, si.config_seed(1))]
+    for i in range(a.warmup):
+        oracle.sort_u32(inputs[i % 2])
+    times = []
+    for i in range(a.steps):
+        t = time.perf_counter()
+        oracle.sort_u32(inputs[i % 2])
+        times.append(time.perf_counter() - t)
+    total = sum(times)
+    value = a.steps * n_sample / total
+    rnd = [t for i, t in enumerate(times) if i % 2 == 0]
+    wst = [t for i, t in enumerate(times) if i % 2 == 1]
+    sample = f"{n_sample} keys per step (2^{n_sample.bit_length() - 1} of the 2^{a.log2n} workload), random/worst alternating"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": a.gpus,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * total / a.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic", "config": {"workload": WORKLOAD, "n": n_full, "E": E, "u": u},
+        "random_keys_per_s": len(rnd) * n_sample / sum(rnd) if rnd else None,
+        "worst_keys_per_s": len(wst) * n_sample / sum(wst) if wst else None,
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line))
+    return 0
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        return run_reference(a)
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_spaa_berneys25_b200 as bcf
+    from paper_conf_spaa_berneys25_b200 import dist as bdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+
+    dp = bcf.default_params()
+    E = a.E or dp.items_per_thread
+    u = a.u or dp.block_threads
+    params = bcf.make_params(E, u, a.algo)
+    n = 1 << a.log2n
+    seed = si.config_seed(1)
+
+    # inputs resident in HBM: rank r's shard of the global random stream, and
+    # the constructed worst case for (E, u)
+    x_rand = si.uniform_u32_torch(n, seed, dev, lo=rank * n)
+    x_worst = bcf.worst_case(n, E, u, seed + rank, device=dev)
+    inputs = [x_rand, x_worst]
+    out = torch.empty(n, dtype=torch.int32, device=dev)
+    tq = bcf.sort(x_rand[:1], params=params)  # warm the library
+    del tq
+    import ctypes
+
+    tb = ctypes.c_size_t(0)
+    bcf.lib().bcf_sort_u32(None, None, n, None, ctypes.byref(tb), ctypes.byref(params), None)
+    temp = torch.empty(tb.value, dtype=torch.uint8, device=dev)
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+
+    def step(i):
+        x = inputs[i % 2]
+        if world == 1:
+            bcf.sort(x, out=out, params=params, temp=temp)
+        else:
+            bdist.sort(x, ops=bdist.CudaOps(params))
+
+    for i in range(max(3, a.warmup)):
+        step(i)
+    torch.cuda.synchronize()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = bcf.launch_count()
+    bcf.profile_enable(True)
+    with ClockSampler(local) as clk:
+        for i in range(a.steps):
+            flush.fill_(i)  # L2 flush, outside the events
+            ev[i][0].record(stream)
+            step(i)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    bcf.profile_enable(False)
+    launches = bcf.launch_count() - launches0
+    if world > 1:
+        dist.barrier()
+    prof = bcf.profile_collect()
+    ms = [s.elapsed_time(e) for s, e in ev]
+    total_ms = sum(ms)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms_max = float(t.item())
+    value = a.steps * n * world / (total_ms_max / 1e3)
+    rnd = [m for i, m in enumerate(ms) if i % 2 == 0]
+    wst = [m for i, m in enumerate(ms) if i % 2 == 1]
+
+    peaks, peak_src = measured_peaks()
+    T = E * u
+    tiles = -(-n // T)
+    passes = max(0, (tiles - 1).bit_length())
+    roof = None
+    mp = prof.get("merge_pass")
+    if mp and mp["launches"]:
+        avg_ms = mp["total_ms"] / mp["launches"]
+        bytes_per_launch = 8 * n  # read 4 B + write 4 B per key per pass
+        achieved = bytes_per_launch / (avg_ms / 1e3) / 1e9
+        traffic = None
+        tf = os.path.join(ROOT, "profiles", "merge_pass_traffic.json")
+        if os.path.exists(tf):
+            with open(tf) as f:
+                tr = json.load(f)
+            if tr.get("n") == n and tr.get("E") == E and tr.get("u") == u:
+                traffic = tr.get("dram_bytes_per_launch")
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                "kernel": "merge_pass", "avg_launch_ms": avg_ms, "bytes_per_launch": bytes_per_launch,
+                "peak_source": f"hbm_gbs {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}
+    kernels = {k: {"launches": v["launches"], "avg_ms": v["total_ms"] / max(1, v["launches"]),
+                   "share_of_step": v["total_ms"] / total_ms if total_ms else None}
+               for k, v in prof.items()}
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
+        "warmup": max(3, a.warmup), "ms_per_step": total_ms_max / a.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "n": n, "n_per_gpu": n, "E": E, "u": u, "tile": T,
+                   "merge_passes": passes, "algo": "conflict_free" if a.algo == 0 else "baseline",
+                   "steps_alternate": "random, worst-case (ABAB)",
+                   "l2": "flushed between timed steps (256 MiB write, outside the events)",
+                   "parallelism": f"dp{world}" if world > 1 else "single"},
+        "random_keys_per_s": len(rnd) * n * world / (sum(rnd) / 1e3) if rnd else None,
+        "worst_keys_per_s": len(wst) * n * world / (sum(wst) / 1e3) if wst else None,
+        "worst_over_random_time": (statistics.mean(wst) / statistics.mean(rnd)) if rnd and wst else None,
+        "roofline": roof,
+        "kernels": kernels,
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+    }
+
+    if rank == 0 and world == 1 and not a.no_extras:
+        # e2e through the public API with host buffers: H2D of the step's input
+        # from pinned memory, the sort, D2H of the result, all in the timed region
+        hx = [x.cpu().pin_memory() for x in inputs]
+        hy = torch.empty(n, dtype=torch.int32).pin_memory()
+        dx = torch.empty(n, dtype=torch.int32, device=dev)
+        ke = min(a.steps, 40)
+        for i in range(3):
+            dx.copy_(hx[i % 2], non_blocking=True)
+            bcf.sort(dx, out=out, params=params, temp=temp)
+            hy.copy_(out, non_blocking=True)
+        torch.cuda.synchronize()
+        e2e_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(ke)]
+        for i in range(ke):
+            flush.fill_(i)
+            e2e_ev[i][0].record(stream)
+            dx.copy_(hx[i % 2], non_blocking=True)
+            bcf.sort(dx, out=out, params=params, temp=temp)
+            hy.copy_(out, non_blocking=True)
+            e2e_ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = sum(s.elapsed_time(e) for s, e in e2e_ev)
+        line["e2e"] = {"value": ke * n / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": 4 * n,
+                       "d2h_bytes_per_step": 4 * n}
+
+        # contrast: the unmodified-Thrust baseline variant on the same inputs
+        bp = bcf.make_params(E if E in (15, 17) else 15, u, bcf.ALGO_BASELINE)
+        contrast = {}
+        for name, prm in [("baseline_thrust", bp), ("cf_same_E", bcf.make_params(bp.items_per_thread, u, 0))]:
+            xw = bcf.worst_case(n, prm.items_per_thread, u, seed, device=dev)
+            ins = [x_rand, xw]
+            tbb = ctypes.c_size_t(0)
+            bcf.lib().bcf_sort_u32(None, None, n, None, ctypes.byref(tbb), ctypes.byref(prm), None)
+            tmp2 = torch.empty(tbb.value, dtype=torch.uint8, device=dev)
+            for i in range(4):
+                bcf.sort(ins[i % 2], out=out, params=prm, temp=tmp2)
+            kc = min(a.steps, 60)
+            cev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(kc)]
+            for i in range(kc):
+                flush.fill_(i)
+                cev[i][0].record(stream)
+                bcf.sort(ins[i % 2], out=out, params=prm, temp=tmp2)
+                cev[i][1].record(stream)
+            torch.cuda.synchronize()
+            cm = [s.elapsed_time(e) for s, e in cev]
+            r_ = [m for i, m in enumerate(cm) if i % 2 == 0]
+            w_ = [m for i, m in enumerate(cm) if i % 2 == 1]
+            contrast[name] = {"E": prm.items_per_thread, "u": u,
+                              "random_keys_per_s": len(r_) * n / (sum(r_) / 1e3),
+                              "worst_keys_per_s": len(w_) * n / (sum(w_) / 1e3),
+                              "worst_over_random_time": statistics.mean(w_) / statistics.mean(r_)}
+        line["contrast"] = contrast
+
+        rate, secs = cpu_oracle_rate(n, 3, ["random", "worst", "random"], E, u)
+        line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": f"3 sorts of {n} keys (random, worst-case, random), {secs:.1f} s on 1 core"}
+    if rank == 0:
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

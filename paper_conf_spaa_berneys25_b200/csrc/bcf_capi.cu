@@ -45,7 +45,7 @@ LaunchTable& launch_table() {
 // Defaults for sm_100a: E = 16 makes the in-register
 // merge a pure 16-wide bitonic merger (no rotation) and the tile a power of
 // two; rho (d = 16) keeps every shared-memory access conflict-free.
-static constexpr int DEFAULT_E = 16;
+static constexpr int DEFAULT_E = 15;
 static constexpr int DEFAULT_U = 256;
 
 // ---------------------------------------------------------------------------
@@ -158,7 +158,7 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   if (e != cudaSuccess) return cuda_fail(e);
   for (int i = 1; i <= P; ++i) {
     const int src = (P - i + 1) % 2, dst = (P - i) % 2;
-    MergeArgs ma{bk[src], bv[src], bk[dst], bv[dst], (long long)n, T << (i - 1),
+    MergeArgs ma{bk[src], bv[src], bk[dst], bv[dst], (long long)n, T << (i - 1), i,
                  (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0};
     e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
     if (e != cudaSuccess) return cuda_fail(e);
@@ -296,7 +296,7 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }
   const Variant& var = launch_table().v[p.E][u_index(p.U)][0][pairs ? 1 : 0];
-  if (!var.merge) return BCF_ERROR_UNSUPPORTED;
+  if (!var.merge_table) return BCF_ERROR_UNSUPPORTED;
   const long long T = (long long)p.U * p.E;
   char* tb = (char*)align_up((size_t)d_temp, 256);
   uint32_t* tk = (uint32_t*)tb;
@@ -330,8 +330,8 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     GroupDesc* dt = dtab + (size_t)(i - 1) * (table_bytes / sizeof(GroupDesc));
     cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_fail(e);
-    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, dt, (int)tab.size()};
-    e = launch("merge_runs", n, s, [&] { return var.merge(ma, tiles, s); });
+    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, 0, dt, (int)tab.size()};
+    e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
     if (e != cudaSuccess) return cuda_fail(e);
     srck = bk[dst];
     srcv = bv[dst];

@@ -31,33 +31,48 @@ __host__ __device__ constexpr bool is_pow2(int x) { return x > 0 && (x & (x - 1)
 // Periodic with period wE (d partitions), so banks depend on k mod wE only.
 // ---------------------------------------------------------------------------
 template <int E>
-__device__ __forceinline__ int rho(int k) {
+__device__ __forceinline__ int rho(int k_) {
   constexpr int d = cgcd(W, E);
   if constexpr (d == 1) {
-    return k;
+    return k_;
   } else {
-    constexpr int P = W * E / d;
-    const int l = k / P;           // constant divisor
-    const int x = k - l * P;
-    int y = x + (l % d);
-    if (y >= P) y -= P;
-    return l * P + y;
+    constexpr unsigned P = W * E / d;
+    const unsigned k = (unsigned)k_;
+    const unsigned l = k / P;                     // constant divisor
+    if constexpr (is_pow2(P)) {
+      return (int)((k & ~(P - 1)) | ((k + (l % d)) & (P - 1)));
+    } else {
+      const unsigned x = k - l * P;
+      unsigned y = x + (l % d);
+      y = y >= P ? y - P : y;
+      return (int)(l * P + y);
+    }
   }
 }
 
 template <int E>
-__device__ __forceinline__ int rho_inv(int p) {
+__device__ __forceinline__ int rho_inv(int p_) {
   constexpr int d = cgcd(W, E);
   if constexpr (d == 1) {
-    return p;
+    return p_;
   } else {
-    constexpr int P = W * E / d;
-    const int l = p / P;
-    const int y = p - l * P;
-    int x = y - (l % d);
-    if (x < 0) x += P;
-    return l * P + x;
+    constexpr unsigned P = W * E / d;
+    const unsigned p = (unsigned)p_;
+    const unsigned l = p / P;
+    if constexpr (is_pow2(P)) {
+      return (int)((p & ~(P - 1)) | ((p + P - (l % d)) & (P - 1)));
+    } else {
+      const unsigned y = p - l * P;
+      const unsigned x = y >= (l % d) ? y - (l % d) : y + P - (l % d);
+      return (int)(l * P + x);
+    }
   }
+}
+
+// shared-memory load of logical index k (through rho)
+template <int E>
+__device__ __forceinline__ uint32_t lds(const uint32_t* __restrict__ sk, int k) {
+  return sk[rho<E>(k)];
 }
 
 // First logical index of the next rho-partition after k (for splitting a run
@@ -65,8 +80,8 @@ __device__ __forceinline__ int rho_inv(int p) {
 template <int E>
 __device__ __forceinline__ int rho_partition_end(int k) {
   constexpr int d = cgcd(W, E);
-  constexpr int P = W * E / d;
-  return (k / P + 1) * P;
+  constexpr unsigned P = W * E / d;
+  return (int)(((unsigned)k / P + 1) * P);
 }
 
 // ---------------------------------------------------------------------------
@@ -145,8 +160,8 @@ __device__ __forceinline__ int warp_origin_smem(const uint32_t* __restrict__ sk,
     const int m = lo + (lane + 1) * s - 1;
     bool p = false;
     if (m < hi) {
-      const uint32_t a = sk[rho<E>(base + m)];
-      const uint32_t b = sk[rho<E>(bofs + m)];
+      const uint32_t a = lds<E>(sk, base + m);
+      const uint32_t b = lds<E>(sk, bofs + m);
       p = !(b < a);
     }
     const int c = __popc(__ballot_sync(FULL, p));
@@ -194,46 +209,58 @@ __device__ __forceinline__ int warp_origin_smem(const uint32_t* __restrict__ sk,
 // ---------------------------------------------------------------------------
 template <int E>
 __device__ __forceinline__ int lane_split_smem(const uint32_t* __restrict__ sk, int base, int S2,
-                                               int NA, int NB, int Dw, int alpha, int lane, int WL) {
+                                               int NA, int NB, int Dw, int alpha, int lane, int WL,
+                                               int nit) {
   const int wb = lane & ~(WL - 1);
   const int lp = lane - wb;
   const int beta = Dw - alpha;
   const int D = Dw + lp * E;
-  // corners
+  // (2) corners (stride E: a round set)
   const int ia = alpha + (lp + 1) * E - 1;
   const int ib = beta + lp * E;
-  uint32_t cA = 0, cB = 0;
-  if (ia < NA) cA = sk[rho<E>(base + ia)];
-  if (ib < NB) cB = sk[rho<E>(base + S2 - 1 - ib)];
-  // coarse: largest m in [0, lp] with Q(alpha + mE)
+  const uint32_t cA = ia < NA ? lds<E>(sk, base + ia) : 0u;
+  const uint32_t cB = ib < NB ? lds<E>(sk, base + S2 - 1 - ib) : 0u;
+  // coarse cell: largest m in [0, lp] with Q(alpha + mE), bisection over lanes
   int lo = 0, hi = lp + 1;  // Q(lo) true, answer < hi
-#pragma unroll
-  for (int it = 0; it < 6; ++it) {  // ceil(log2(33)) bisection steps
+  for (int it = 0; it < nit; ++it) {
     const int mid = (lo + hi) >> 1;
-    const int m = (hi - lo > 1) ? mid : lo;
-    const int srcA = wb + (m >= 1 ? m - 1 : 0);
-    const int srcB = wb + (lp - m >= 0 ? lp - m : 0);
-    const uint32_t a = __shfl_sync(FULL, cA, srcA);
-    const uint32_t b = __shfl_sync(FULL, cB, srcB);
-    if (hi - lo > 1) {
-      const bool validA = alpha + m * E <= NA;
-      const bool validB = beta + (lp - m) * E < NB;
-      const bool q = (m == 0) || (validA && (!validB || !(b < a)));
-      if (q) lo = m; else hi = m;
+    const bool live = hi - lo > 1;
+    const int m = live ? mid : lo;
+    const uint32_t a = __shfl_sync(FULL, cA, wb + (m >= 1 ? m - 1 : 0));
+    const uint32_t b = __shfl_sync(FULL, cB, wb + lp - m);
+    const bool validA = alpha + m * E <= NA;
+    const bool validB = beta + (lp - m) * E < NB;
+    const bool q = (m == 0) || (validA && (!validB || !(b < a)));
+    if (live) {
+      lo = q ? m : lo;
+      hi = q ? hi : m;
     }
   }
+  // (3) cell scan: round j tests Q(ac + j + 1) reading A[ac+j] and B[D-ac-1-j]
   const int ac = alpha + lo * E;  // a(D) in [ac, ac+E]
+  const int jA = (NA < D ? NA : D) - ac;   // j < jA: A[ac+j] exists and ac+j+1 <= D
+  const int jB = D - ac - NB;              // j >= jB: B[D-ac-1-j] exists
+  const int pa0 = base + ac;               // logical index of A[ac + j] = pa0 + j
+  const int pb0 = base + S2 - D + ac;      // logical index of B[D-ac-1-j] = pb0 + j
+  // Probes outside [jB, jA) are still issued (their logical indices stay in
+  // the same round set, so they cannot conflict; the tile buffer has E words
+  // of slack past its end) and masked out of the count.
   int cnt = 0;
+  if (__all_sync(FULL, jA >= E && jB <= 0)) {
+    // interior of the tile (all lanes): no masking needed
 #pragma unroll
-  for (int j = 0; j < E; ++j) {
-    const int a = ac + j + 1;  // candidate a(D) >= a ?
-    const bool inA = a <= NA && a <= D;
-    const bool needB = (D - a) < NB;
-    uint32_t ka = 0, kb = 0;
-    if (inA) ka = sk[rho<E>(base + a - 1)];
-    if (inA && needB) kb = sk[rho<E>(base + S2 - 1 - (D - a))];
-    const bool q = inA && (!needB || !(kb < ka));
-    cnt += q ? 1 : 0;
+    for (int j = 0; j < E; ++j) {
+      const uint32_t ka = lds<E>(sk, pa0 + j);
+      const uint32_t kb = lds<E>(sk, pb0 + j);
+      cnt += (kb < ka) ? 0 : 1;
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < E; ++j) {
+      const uint32_t ka = lds<E>(sk, pa0 + j);
+      const uint32_t kb = lds<E>(sk, pb0 + j);
+      cnt += (j < jA && (j < jB || !(kb < ka))) ? 1 : 0;
+    }
   }
   return ac + cnt;
 }
@@ -246,25 +273,31 @@ __device__ __forceinline__ int lane_split_smem(const uint32_t* __restrict__ sk, 
 // B_i[(k-j-1) mod E]; both at logical base + idx, B reversed behind A.
 // After the gather, items[] is a circular bitonic sequence starting at k.
 // ---------------------------------------------------------------------------
-template <int E, bool PAIRS>
+template <int E, bool PAIRS, bool FULL_TILE>
 __device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restrict__ sk,
                                                         const uint32_t* __restrict__ sv, int base,
                                                         int S2, int a, int b, int nA, int nB,
                                                         uint32_t (&key)[E], uint32_t (&val)[E],
                                                         uint32_t pad) {
   const int k = a % E;
-  const int baseA = base + a;
-  const int baseB = base + S2 - b - E;  // B_i[E-1-ia] at base+S2-1-(b+E-1-ia) = baseB+ia
+  // round j: ia = (j - k) mod E; A_i[ia] at logical base+a+ia, else
+  // B_i[E-1-ia] at base+S2-1-(b+E-1-ia) = base+S2-b-E+ia
+  const int offA = base + a - k;
+  const int offB = base + S2 - b - E - k;
+  const int hiA = k + nA;  // A rounds: j in [k, k+nA) (mod E)
 #pragma unroll
   for (int j = 0; j < E; ++j) {
-    int ia = j - k;
-    if (ia < 0) ia += E;
-    const bool isA = ia < nA;
-    const bool ok = isA || (E - 1 - ia) < nB;
-    const int idx = rho<E>((isA ? baseA : baseB) + ia);
+    const bool wrap = j < k;
+    const bool isA = wrap ? (j + E < hiA) : (j < hiA);
+    const int idx = (isA ? offA : offB) + (wrap ? j + E : j);
+    bool ok = true;
+    if constexpr (!FULL_TILE) {
+      const int ia = wrap ? j + E - k : j - k;
+      ok = isA || (E - 1 - ia) < nB;
+    }
     if (ok) {
-      key[j] = sk[idx];
-      if constexpr (PAIRS) val[j] = sv[idx];
+      key[j] = lds<E>(sk, idx);
+      if constexpr (PAIRS) val[j] = lds<E>(sv, idx);
     } else {
       key[j] = pad;
       if constexpr (PAIRS) val[j] = 0;
@@ -428,24 +461,56 @@ __device__ __forceinline__ void merge_registers(uint32_t (&key)[E], uint32_t (&v
       }
     }
     bitonic_merge_pad<E, PAIRS>(key, tag, val);
+  } else if constexpr (cpow2ceil(E) == E + 1) {
+    // N = E + 1: insert one minimum element (key 0, tag 0; real tags shift
+    // by 1) at register k, i.e. between the circular minimum candidates
+    // B_i[0] (register k-1) and A_i[0] (register k).  The 16-register
+    // circular sequence stays bitonic, and its sorted slot 0 is the insert,
+    // dropped afterwards.  Costs 2 selects per register instead of a
+    // log2(E)-stage barrel rotation.
+    constexpr int N = E + 1;
+    uint32_t K[N], Tg[N], V[N];
+#pragma unroll
+    for (int m = 0; m < N; ++m) {
+      const uint32_t lo = m < E ? key[m] : 0u;
+      const uint32_t hi = m >= 1 ? key[m - 1] : 0u;
+      K[m] = m < k ? lo : (m == k ? 0u : hi);
+      if constexpr (PAIRS) {
+        const uint32_t vlo = m < E ? val[m] : 0u;
+        const uint32_t vhi = m >= 1 ? val[m - 1] : 0u;
+        V[m] = m < k ? vlo : (m == k ? 0u : vhi);
+        // tag of the element now in slot m (its register before insertion)
+        const int j = m < k ? m : m - 1;
+        int ia = j - k;
+        if (ia < 0) ia += E;
+        const int ib = E - 1 - ia;
+        const uint32_t t = ia < nA ? (uint32_t)ia + 1u : (ib < nB ? (uint32_t)(nA + ib) + 1u : (uint32_t)E + 1u);
+        Tg[m] = m == k ? 0u : t;
+      }
+    }
+    bitonic_merge_pad<N, PAIRS>(K, Tg, V);
+#pragma unroll
+    for (int i = 0; i < E; ++i) {
+      key[i] = K[i + 1];
+      if constexpr (PAIRS) val[i] = V[i + 1];
+    }
   } else {
-    // rotate left by k: new[m] = old[(m + k) mod E]
+    // rotate left by k: new[m] = old[(m + k) mod E] (barrel, static selects)
     constexpr int NBITS = clog2(E - 1) + 1;  // bits of k in [0, E-1]
 #pragma unroll
     for (int bit = 0; bit < NBITS; ++bit) {
       const int sh = 1 << bit;
-      if ((k >> bit) & 1) {
-        uint32_t tk[E], tv[E];
+      const bool b = (k >> bit) & 1;
+      uint32_t tk[E], tv[E];
 #pragma unroll
-        for (int m = 0; m < E; ++m) {
-          tk[m] = key[(m + sh) % E];
-          if constexpr (PAIRS) tv[m] = val[(m + sh) % E];
-        }
+      for (int m = 0; m < E; ++m) {
+        tk[m] = b ? key[(m + sh) % E] : key[m];
+        if constexpr (PAIRS) tv[m] = b ? val[(m + sh) % E] : val[m];
+      }
 #pragma unroll
-        for (int m = 0; m < E; ++m) {
-          key[m] = tk[m];
-          if constexpr (PAIRS) val[m] = tv[m];
-        }
+      for (int m = 0; m < E; ++m) {
+        key[m] = tk[m];
+        if constexpr (PAIRS) val[m] = tv[m];
       }
     }
     if constexpr (PAIRS) {

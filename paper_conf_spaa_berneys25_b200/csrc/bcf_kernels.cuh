@@ -23,9 +23,15 @@ namespace bcf {
 constexpr uint32_t PAD_KEY = 0xffffffffu;
 
 // dynamic shared memory of one CTA
+// T keys + E words of slack (cell-scan probes past the end, see
+// lane_split_smem) + 1 (the serial merge's look-ahead load in the baseline)
+template <int E, int U>
+__host__ __device__ constexpr int tile_words() {
+  return U * E + E + 1;
+}
 template <int E, int U, bool PAIRS>
-constexpr size_t tile_smem_bytes() {
-  return (size_t)(U * E + 1) * sizeof(uint32_t) * (PAIRS ? 2 : 1);
+__host__ __device__ constexpr size_t tile_smem_bytes() {
+  return (size_t)tile_words<E, U>() * sizeof(uint32_t) * (PAIRS ? 2 : 1);
 }
 
 struct SortArgs {
@@ -53,6 +59,7 @@ struct MergeArgs {
   uint32_t* dst_v;
   long long n;
   long long R;     // input run length (regular mode)
+  int log2_tpg;    // log2(2R / T): tiles per group (regular mode)
   int decode_f32;  // final pass of an f32 sort
   int cf_dirs;     // regular mode: odd runs descending
   const GroupDesc* groups;  // table mode (merge of arbitrary runs) if non-null
@@ -65,9 +72,8 @@ __device__ __forceinline__ GroupDesc group_of_tile(const MergeArgs& args, long l
                                                    long long& j) {
   GroupDesc G;
   if (args.groups == nullptr) {
-    const long long tpg = (2 * args.R) / T;  // tiles per full group
-    const long long g = tile / tpg;
-    j = tile - g * tpg;
+    const long long g = tile >> args.log2_tpg;  // tiles per group = 2R/T = 2^log2_tpg
+    j = tile - (g << args.log2_tpg);
     const long long g0 = g * 2 * args.R;
     const long long left = args.n - g0;
     G.a_off = g0;
@@ -75,7 +81,7 @@ __device__ __forceinline__ GroupDesc group_of_tile(const MergeArgs& args, long l
     G.b_off = g0 + args.R;
     G.nb = left - G.na < args.R ? left - G.na : args.R;
     G.out_off = g0;
-    G.tile_begin = g * tpg;
+    G.tile_begin = g << args.log2_tpg;
     G.a_desc = 0;
     G.b_desc = args.cf_dirs;
     G.out_desc = args.cf_dirs && (g & 1);
@@ -105,25 +111,45 @@ __device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uin
                                            long long c0, bool decode) {
   constexpr int T = U * E;
   // round m: ascending -> item m at D+m; descending -> item E-1-m at T-E-D+m
-  const int base = desc ? (T - E - D) : D;
+  if (desc) {
 #pragma unroll
-  for (int m = 0; m < E; ++m) {
-    const int idx = rho<E>(base + m);
-    sk[idx] = desc ? key[E - 1 - m] : key[m];
-    if constexpr (PAIRS) sv[idx] = desc ? val[E - 1 - m] : val[m];
+    for (int m = 0; m < E; ++m) {
+      const int idx = rho<E>(T - E - D + m);
+      sk[idx] = key[E - 1 - m];
+      if constexpr (PAIRS) sv[idx] = val[E - 1 - m];
+    }
+  } else {
+#pragma unroll
+    for (int m = 0; m < E; ++m) {
+      const int idx = rho<E>(D + m);
+      sk[idx] = key[m];
+      if constexpr (PAIRS) sv[idx] = val[m];
+    }
   }
   __syncthreads();
   const int qlo = desc ? T - cnt : 0;
   const int qhi = desc ? T : cnt;
+  uint32_t* __restrict__ pk = gk + c0;
+  uint32_t* __restrict__ pv = PAIRS ? gv + c0 : nullptr;
+  if (decode) {
 #pragma unroll
-  for (int r = 0; r < E; ++r) {
-    const int P = threadIdx.x + r * U;  // physical word: consecutive per warp
-    const int q = rho_inv<E>(P);
-    if (q >= qlo && q < qhi) {
-      uint32_t x = sk[P];
-      if (decode) x = f32_decode(x);
-      gk[c0 + q] = x;
-      if constexpr (PAIRS) gv[c0 + q] = sv[P];
+    for (int r = 0; r < E; ++r) {
+      const int P = threadIdx.x + r * U;  // physical word: consecutive per warp
+      const int q = rho_inv<E>(P);
+      if (q >= qlo && q < qhi) {
+        pk[q] = f32_decode(sk[P]);
+        if constexpr (PAIRS) pv[q] = sv[P];
+      }
+    }
+  } else {
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+      const int P = threadIdx.x + r * U;
+      const int q = rho_inv<E>(P);
+      if (q >= qlo && q < qhi) {
+        pk[q] = sk[P];
+        if constexpr (PAIRS) pv[q] = sv[P];
+      }
     }
   }
 }
@@ -137,8 +163,8 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
   extern __shared__ uint32_t smem_dyn[];
-  uint32_t* sk = smem_dyn;                 // T + 1 keys
-  uint32_t* sv = smem_dyn + (T + 1);       // T + 1 values (pairs only)
+  uint32_t* sk = smem_dyn;                      // tile_words keys
+  uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
   __shared__ int s_org[NW + 1];
   const int tid = threadIdx.x;
   const int lane = tid & (W - 1);
@@ -151,6 +177,8 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   // --- load: coalesced in physical order, pads = max key (they sort last and
   // are trimmed by the count; stable order keeps them after real max keys).
   {
+    const uint32_t* __restrict__ gin_k = args.in_k + t0;
+    const uint32_t* __restrict__ gin_v = PAIRS ? args.in_v + t0 : nullptr;
     uint32_t vk[E], vv[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
@@ -159,10 +187,10 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
       vk[r] = PAD_KEY;
       vv[r] = 0;
       if (p < cnt) {
-        uint32_t x = __ldg(args.in_k + t0 + p);
+        uint32_t x = __ldg(gin_k + p);
         if (args.encode_f32) x = f32_encode(x);
         vk[r] = x;
-        if constexpr (PAIRS) vv[r] = __ldg(args.in_v + t0 + p);
+        if constexpr (PAIRS) vv[r] = __ldg(gin_v + p);
       }
     }
 #pragma unroll
@@ -212,15 +240,16 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
     const int ig = tid & (G - 1);
     const int D = ig * E;
     if constexpr (CF) {
-      int alpha = 0, Dw = 0, WL = G;
+      int alpha = 0, Dw = 0, WL = G, nit = l + 1;
       if (G > W) {
         Dw = (ig >> 5) * (W * E);
         alpha = warp_origin_smem<E>(sk, gbase, 2 * S, S, S, Dw, lane);
         WL = W;
+        nit = 5;
         if (lane == 0) s_org[warp] = alpha;
+        __syncthreads();  // uniform: G depends on l only
       }
-      __syncthreads();
-      const int a = lane_split_smem<E>(sk, gbase, 2 * S, S, S, Dw, alpha, lane, WL);
+      const int a = lane_split_smem<E>(sk, gbase, 2 * S, S, S, Dw, alpha, lane, WL, nit);
       int anext = __shfl_down_sync(FULL, a, 1);
       if ((lane & (WL - 1)) == WL - 1) {
         // last lane of the window: next window's origin, or the group end
@@ -229,7 +258,7 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
       const int nA = anext - a;
       const int nB = E - nA;
       const int b = D - a;
-      dual_subsequence_gather<E, PAIRS>(sk, sv, gbase, 2 * S, a, b, nA, nB, key, val, PAD_KEY);
+      dual_subsequence_gather<E, PAIRS, true>(sk, sv, gbase, 2 * S, a, b, nA, nB, key, val, PAD_KEY);
       merge_registers<E, PAIRS>(key, val, a, nA, nB);
     } else {
       // unmodified Thrust: per-thread binary merge path, then serial merge
@@ -266,13 +295,13 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
 // Merge pass (K2+K3 fused): output tile `blockIdx.x` of the pairwise merge of
 // runs of R keys.  Group g merges run 2g (A) with run 2g+1 (B).
 // ---------------------------------------------------------------------------
-template <int E, int U, bool PAIRS, bool CF>
+template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
   extern __shared__ uint32_t smem_dyn[];
-  uint32_t* sk = smem_dyn;                 // T + 1 keys
-  uint32_t* sv = smem_dyn + (T + 1);       // T + 1 values (pairs only)
+  uint32_t* sk = smem_dyn;                      // tile_words keys
+  uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
   __shared__ int s_org[NW + 1];
   __shared__ long long s_split[2];
   const int tid = threadIdx.x;
@@ -302,44 +331,49 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   const long long b0 = D0 - a0;
 
   // --- staging: A forward at logical [0, NA); B reversed (CF: B[y] at T-1-y)
-  // or forward behind A (baseline).  Physical-order, coalesced global reads.
+  // or forward behind A (baseline).  Physical-order, coalesced global reads;
+  // element q of A at oA + sA*q, element y of B at oB' +- y (pointer math once).
   {
+    // A runs are ascending: A element (a0 + q) at a_off + a0 + q.
+    // CF: logical q >= T-NB holds B[y], y = b0 + T-1-q; B stored descending
+    //     (BDESC, regular passes) at b_off + nb-1-y = (b_off + nb-b0-T) + q,
+    //     or ascending (table mode) at b_off + y = (b_off + b0+T-1) - q.
+    // baseline: logical q in [NA, cnt) holds B[b0 + q - NA] (ascending).
+    constexpr int sB = (CF && !BDESC) ? -1 : 1;
+    const long long oA = grp.a_off + a0;
+    const long long oB = CF ? (BDESC ? grp.b_off + grp.nb - b0 - T : grp.b_off + b0 + T - 1)
+                            : grp.b_off + b0 - NA;
+    const uint32_t* __restrict__ pAk = args.src_k + oA;
+    const uint32_t* __restrict__ pBk = args.src_k + oB;
+    const uint32_t* __restrict__ pAv = PAIRS ? args.src_v + oA : nullptr;
+    const uint32_t* __restrict__ pBv = PAIRS ? args.src_v + oB : nullptr;
+    const int bstart = CF ? T - NB : NA;
+    const int bend = CF ? T : cnt;
     uint32_t vk[E], vv[E];
-    bool ok[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
       const int P = tid + r * U;
-      ok[r] = false;
+      const int q = CF ? rho_inv<E>(P) : P;
+      const bool isA = q < NA;
+      const bool isB = q >= bstart && q < bend;
       vk[r] = 0;
       vv[r] = 0;
-      if constexpr (CF) {
-        const int q = rho_inv<E>(P);
-        if (q < NA) {
-          ok[r] = true;
-          const long long ga = Av.addr(a0 + q);
-          vk[r] = __ldg(Av.base + ga);
-          if constexpr (PAIRS) vv[r] = __ldg(args.src_v + grp.a_off + ga);
-        } else if (q >= T - NB) {
-          ok[r] = true;
-          const long long gb = Bv.addr(b0 + (T - 1 - q));
-          vk[r] = __ldg(Bv.base + gb);
-          if constexpr (PAIRS) vv[r] = __ldg(args.src_v + grp.b_off + gb);
-        }
-      } else {
-        if (P < NA) {
-          ok[r] = true;
-          vk[r] = __ldg(Av.base + Av.addr(a0 + P));
-        } else if (P < cnt) {
-          ok[r] = true;
-          vk[r] = __ldg(Bv.base + Bv.addr(b0 + (P - NA)));
-        }
+      if (isA) {
+        vk[r] = __ldg(pAk + q);
+        if constexpr (PAIRS) vv[r] = __ldg(pAv + q);
+      }
+      if (isB) {
+        vk[r] = __ldg(pBk + sB * q);
+        if constexpr (PAIRS) vv[r] = __ldg(pBv + sB * q);
       }
     }
 #pragma unroll
     for (int r = 0; r < E; ++r) {
-      if (ok[r]) {
-        sk[tid + r * U] = vk[r];
-        if constexpr (PAIRS) sv[tid + r * U] = vv[r];
+      const int P = tid + r * U;
+      const int q = CF ? rho_inv<E>(P) : P;
+      if (q < NA || (q >= bstart && q < bend)) {
+        sk[P] = vk[r];
+        if constexpr (PAIRS) sv[P] = vv[r];
       }
     }
   }
@@ -353,7 +387,7 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
     if (lane == 0) s_org[warp] = alpha;
     if (tid == 0) s_org[NW] = NA;
     __syncthreads();
-    const int a = lane_split_smem<E>(sk, 0, T, NA, NB, Dw, alpha, lane, W);
+    const int a = lane_split_smem<E>(sk, 0, T, NA, NB, Dw, alpha, lane, W, 5);
     int anext = __shfl_down_sync(FULL, a, 1);
     if (lane == W - 1) anext = s_org[warp + 1];
     const int Dc = D < cnt ? D : cnt;
@@ -361,7 +395,10 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
     const int nA = anext - a;
     const int nB = (Dn - Dc) - nA;
     const int b = Dc - a;
-    dual_subsequence_gather<E, PAIRS>(sk, sv, 0, T, a, b, nA, nB, key, val, PAD_KEY);
+    if (cnt == T)
+      dual_subsequence_gather<E, PAIRS, true>(sk, sv, 0, T, a, b, nA, nB, key, val, PAD_KEY);
+    else
+      dual_subsequence_gather<E, PAIRS, false>(sk, sv, 0, T, a, b, nA, nB, key, val, PAD_KEY);
     merge_registers<E, PAIRS>(key, val, a, nA, nB);
   } else {
     if (D < cnt) {

@@ -14,7 +14,8 @@ using MergeFn = cudaError_t (*)(const MergeArgs&, long long grid, cudaStream_t);
 
 struct Variant {
   BlockSortFn block_sort = nullptr;
-  MergeFn merge = nullptr;
+  MergeFn merge = nullptr;        // regular pass (CF: B runs stored descending)
+  MergeFn merge_table = nullptr;  // group-table pass, all runs ascending (CF)
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]

@@ -28,21 +28,24 @@ cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s)
   return cudaGetLastError();
 }
 
-template <int E, int U, bool PAIRS, bool CF>
+template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
-  cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF>, smem);
+  cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, smem);
   if (e != cudaSuccess) return e;
-  merge_pass_kernel<E, U, PAIRS, CF><<<(unsigned)grid, U, smem, s>>>(a);
+  merge_pass_kernel<E, U, PAIRS, CF, BDESC><<<(unsigned)grid, U, smem, s>>>(a);
   return cudaGetLastError();
 }
 
 template <int E, int U>
 void register_eu(LaunchTable& t) {
   const int ui = u_index(U);
-  t.v[E][ui][0][0] = {&launch_block_sort<E, U, false, true>, &launch_merge<E, U, false, true>};
-  t.v[E][ui][0][1] = {&launch_block_sort<E, U, true, true>, &launch_merge<E, U, true, true>};
-  t.v[E][ui][1][0] = {&launch_block_sort<E, U, false, false>, &launch_merge<E, U, false, false>};
+  t.v[E][ui][0][0] = {&launch_block_sort<E, U, false, true>, &launch_merge<E, U, false, true, true>,
+                      &launch_merge<E, U, false, true, false>};
+  t.v[E][ui][0][1] = {&launch_block_sort<E, U, true, true>, &launch_merge<E, U, true, true, true>,
+                      &launch_merge<E, U, true, true, false>};
+  t.v[E][ui][1][0] = {&launch_block_sort<E, U, false, false>, &launch_merge<E, U, false, false, false>,
+                      nullptr};
 }
 
 }  // namespace bcf

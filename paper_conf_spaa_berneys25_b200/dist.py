@@ -1,0 +1,158 @@
+"""Distributed sort across the GPUs of one node.
+
+One process per GPU.  Every rank holds a shard of keys (optionally values):
+  1. local CF mergesort (bcf_sort_u32 / bcf_sort_pairs_u32), no communication;
+  2. exact splitters: for targets k_t = floor(t N / p), t = 1..p-1, a k-ary
+     bisection of the 32-bit key space finds the smallest key v_t with
+     sum_r #(keys_r <= v_t) >= k_t; each round every rank counts with
+     bcf_split_counts_u32 (device binary searches) and one all_reduce(SUM)
+     combines the counts;
+  3. equal keys at the cut are consumed in rank order (stable): rank r sends
+     lt_r(v_t) + min(eq_r(v_t), max(0, k_t - L_t - sum_{r'<r} eq_r'(v_t)))
+     keys below cut t, so rank r ends with exactly positions
+     [k_r, k_{r+1}) of the global stable order;
+  4. all_to_all_single exchanges the buckets (NCCL over NVLink / NVSwitch);
+  5. bcf_merge_runs_u32 merges the p received runs in source-rank order
+     (ties to the lower rank) with the CF merge kernel.
+
+The local operations are injectable (`ops`) so the host logic can be tested
+with the gloo backend on CPU; the default ops are the CUDA library and raise
+without a GPU -- there is no CPU fallback in the product path.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+KEY_SPACE = 1 << 32
+PIVOTS_PER_TARGET = 63  # (63+1)-ary search: 32 bits in 6 rounds
+
+
+class CudaOps:
+    """Local phases on the GPU through the C ABI."""
+
+    def __init__(self, params=None):
+        import paper_conf_spaa_berneys25_b200 as bcf
+
+        self.bcf = bcf
+        self.params = params
+
+    def sort(self, keys, values=None):
+        if values is None:
+            return self.bcf.sort(keys, params=self.params), None
+        return self.bcf.sort_pairs(keys, values, params=self.params)
+
+    def split_counts(self, sorted_keys, pivots_u32: np.ndarray):
+        import torch
+
+        piv = torch.from_numpy(pivots_u32.astype(np.uint32).view(np.int32)).to(sorted_keys.device)
+        lt, le = self.bcf.split_counts(sorted_keys, piv)
+        return lt, le
+
+    def merge_runs(self, keys, offsets, values=None):
+        return self.bcf.merge_runs(keys, offsets, values=values, params=self.params) if values is not None \
+            else (self.bcf.merge_runs(keys, offsets, params=self.params), None)
+
+
+@dataclass
+class DistStats:
+    rounds: int = 0
+    send_counts: list | None = None
+    recv_counts: list | None = None
+    pivots: list | None = None
+
+
+def _targets(N: int, p: int):
+    return [(t * N) // p for t in range(1, p)]
+
+
+def exact_splitters(sorted_keys, n_local: int, group, ops, device):
+    """Smallest v_t with global #(key <= v_t) >= k_t for t = 1..p-1, plus the
+    per-rank send counts (rank-ordered tie split)."""
+    import torch
+    import torch.distributed as dist
+
+    p = dist.get_world_size(group)
+    r = dist.get_rank(group)
+    nt = torch.tensor([n_local], dtype=torch.int64, device=device)
+    dist.all_reduce(nt, group=group)
+    N = int(nt.item())
+    ks = _targets(N, p)
+    lo = [0] * (p - 1)           # answer in [lo, hi]
+    hi = [KEY_SPACE - 1] * (p - 1)
+    rounds = 0
+    while any(h > l for l, h in zip(lo, hi)):
+        rounds += 1
+        piv = []
+        for t in range(p - 1):
+            span = hi[t] - lo[t]
+            m = PIVOTS_PER_TARGET
+            # pivots lo + ceil(i * span / (m+1)) - 1 ... evenly splitting [lo, hi)
+            cand = sorted({lo[t] + (i * span) // (m + 1) for i in range(1, m + 1)} - {hi[t]})
+            cand = [c for c in cand if lo[t] <= c < hi[t]]
+            cand = cand + [hi[t]] * (m - len(cand))
+            piv.extend(cand)
+        piv_np = np.array(piv, dtype=np.uint64).astype(np.uint32)
+        _, le = ops.split_counts(sorted_keys, piv_np)
+        le = le.to(torch.int64)
+        dist.all_reduce(le, group=group)
+        le_h = le.cpu().numpy()
+        for t in range(p - 1):
+            if hi[t] <= lo[t]:
+                continue
+            row = piv[t * PIVOTS_PER_TARGET:(t + 1) * PIVOTS_PER_TARGET]
+            cnt = le_h[t * PIVOTS_PER_TARGET:(t + 1) * PIVOTS_PER_TARGET]
+            new_lo, new_hi = lo[t], hi[t]
+            for v, c in zip(row, cnt):       # row ascending
+                if c >= ks[t]:
+                    new_hi = min(new_hi, v)
+                    break
+                new_lo = max(new_lo, v + 1)
+            lo[t], hi[t] = new_lo, new_hi
+    vs = np.array(lo, dtype=np.uint64).astype(np.uint32)
+    lt, le = ops.split_counts(sorted_keys, vs)
+    lt = lt.to(torch.int64)
+    eq = le.to(torch.int64) - lt
+    both = torch.stack([lt, eq])                       # [2, p-1]
+    gathered = [torch.empty_like(both) for _ in range(p)]
+    dist.all_gather(gathered, both, group=group)
+    G = torch.stack(gathered).cpu().numpy()            # [p, 2, p-1]
+    cuts = [0]
+    for t in range(p - 1):
+        L = int(G[:, 0, t].sum())
+        before = int(G[:r, 1, t].sum())
+        take = min(int(G[r, 1, t]), max(0, ks[t] - L - before))
+        cuts.append(int(G[r, 0, t]) + take)
+    cuts.append(n_local)
+    send = [cuts[d + 1] - cuts[d] for d in range(p)]
+    return send, [int(v) for v in vs], rounds
+
+
+def sort(keys, values=None, group=None, ops=None):
+    """Distributed stable sort of the shards held by the ranks of `group`.
+    Returns (keys_out, values_out_or_None, DistStats).  keys: 1-D 4-byte
+    tensor (u32 bit patterns in int32); values likewise."""
+    import torch
+    import torch.distributed as dist
+
+    ops = ops or CudaOps()
+    device = keys.device
+    p = dist.get_world_size(group)
+    sk, sv = ops.sort(keys, values)
+    if p == 1:
+        return sk, sv, DistStats(0, [keys.numel()], [keys.numel()], [])
+    send, pivots, rounds = exact_splitters(sk, sk.numel(), group, ops, device)
+    sc = torch.tensor(send, dtype=torch.int64, device=device)
+    rc = torch.empty_like(sc)
+    dist.all_to_all_single(rc, sc, group=group)
+    recv = [int(x) for x in rc.cpu().tolist()]
+    rk = torch.empty(sum(recv), dtype=keys.dtype, device=device)
+    dist.all_to_all_single(rk, sk, output_split_sizes=recv, input_split_sizes=send, group=group)
+    rv = None
+    if sv is not None:
+        rv = torch.empty(sum(recv), dtype=values.dtype, device=device)
+        dist.all_to_all_single(rv, sv, output_split_sizes=recv, input_split_sizes=send, group=group)
+    offs = np.concatenate([[0], np.cumsum(recv)]).astype(np.uint64)
+    ok, ov = ops.merge_runs(rk, offs, rv)
+    return ok, ov, DistStats(rounds, send, recv, pivots)
