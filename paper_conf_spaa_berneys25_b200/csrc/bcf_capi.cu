@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -113,6 +114,15 @@ static bcf_status resolve(const bcf_params* p, Params& out) {
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+// BCF_NO_TMA=1 selects the non-persistent merge kernel (A/B measurements)
+static bool tma_disabled() {
+  static const bool off = [] {
+    const char* v = getenv("BCF_NO_TMA");
+    return v && v[0] == '1';
+  }();
+  return off;
+}
+
 // ---------------------------------------------------------------------------
 // the pairwise mergesort driver
 //   block sort: tiles of T = U*E -> runs of T (run r descending iff r odd, CF)
@@ -128,8 +138,10 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   bcf_status st = resolve(pp, p);
   if (st != BCF_SUCCESS) return st;
   if (pairs && p.algo == BCF_ALGO_BASELINE) return BCF_ERROR_UNSUPPORTED;
-  const size_t key_bytes = align_up((size_t)n * sizeof(uint32_t), 256);
-  const size_t need = 256 + key_bytes * (pairs ? 2 : 1);
+  // two ping-pong buffers X, Y (256-B aligned, 64 words of slack for the
+  // sigma-shifted descending runs); only the final pass writes d_out
+  const size_t key_bytes = align_up(((size_t)n + 64) * sizeof(uint32_t), 256);
+  const size_t need = 256 + key_bytes * 2 * (pairs ? 2 : 1);
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -146,21 +158,29 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   int P = 0;
   while ((T << P) < (long long)n) ++P;
   const bool cf = p.algo == BCF_ALGO_CONFLICT_FREE;
+  const bool use_tma = cf && var.merge_tma != nullptr && !tma_disabled();
 
   char* tb = (char*)align_up((size_t)d_temp, 256);
-  uint32_t* tk = (uint32_t*)tb;
-  uint32_t* tv = pairs ? (uint32_t*)(tb + key_bytes) : nullptr;
-  uint32_t* bk[2] = {out_k, tk};
-  uint32_t* bv[2] = {out_v, tv};
+  uint32_t* X = (uint32_t*)tb;
+  uint32_t* Y = (uint32_t*)(tb + key_bytes);
+  uint32_t* XV = pairs ? (uint32_t*)(tb + 2 * key_bytes) : nullptr;
+  uint32_t* YV = pairs ? (uint32_t*)(tb + 3 * key_bytes) : nullptr;
 
-  SortArgs sa{in_k, in_v, bk[P % 2], bv[P % 2], (long long)n, f32 ? 1 : 0, (f32 && P == 0) ? 1 : 0, cf ? 1 : 0};
+  SortArgs sa{in_k, in_v, P == 0 ? out_k : X, P == 0 ? out_v : XV, (long long)n, f32 ? 1 : 0,
+              (f32 && P == 0) ? 1 : 0, cf ? 1 : 0};
   cudaError_t e = launch("block_sort", n, s, [&] { return var.block_sort(sa, tiles, s); });
   if (e != cudaSuccess) return cuda_fail(e);
   for (int i = 1; i <= P; ++i) {
-    const int src = (P - i + 1) % 2, dst = (P - i) % 2;
-    MergeArgs ma{bk[src], bv[src], bk[dst], bv[dst], (long long)n, T << (i - 1), i,
+    uint32_t* sk = (i & 1) ? X : Y;
+    uint32_t* sv = (i & 1) ? XV : YV;
+    uint32_t* dk = i == P ? out_k : ((i & 1) ? Y : X);
+    uint32_t* dv = i == P ? out_v : ((i & 1) ? YV : XV);
+    MergeArgs ma{sk, sv, dk, dv, (long long)n, T << (i - 1), i,
                  (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0};
-    e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
+    if (use_tma)
+      e = launch("merge_pass", n, s, [&] { return var.merge_tma(ma, tiles, s); });
+    else
+      e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
     if (e != cudaSuccess) return cuda_fail(e);
   }
   return BCF_SUCCESS;

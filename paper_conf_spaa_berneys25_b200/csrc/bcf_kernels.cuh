@@ -78,13 +78,15 @@ __device__ __forceinline__ GroupDesc group_of_tile(const MergeArgs& args, long l
     const long long left = args.n - g0;
     G.a_off = g0;
     G.na = left < args.R ? left : args.R;
-    G.b_off = g0 + args.R;
     G.nb = left - G.na < args.R ? left - G.na : args.R;
-    G.out_off = g0;
+    // descending runs of length L < R are stored shifted by sigma = (R-L) mod 4
+    // so that a tile's A range and B range share one 16-byte phase (TMA path)
+    G.b_off = g0 + args.R + (args.cf_dirs ? ((args.R - G.nb) & 3) : 0);
     G.tile_begin = g << args.log2_tpg;
     G.a_desc = 0;
     G.b_desc = args.cf_dirs;
     G.out_desc = args.cf_dirs && (g & 1);
+    G.out_off = g0 + (G.out_desc ? ((2 * args.R - G.na - G.nb) & 3) : 0);
   } else {
     int lo = 0, hi = args.ngroups - 1;  // last group with tile_begin <= tile
     while (lo < hi) {
@@ -286,7 +288,8 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   __syncthreads();
   // --- store run `tile`: descending iff tile odd (CF directions)
   const bool desc = args.cf_dirs && (tile & 1);
-  const long long c0 = desc ? t0 + cnt - T : t0;
+  // a short descending run is stored shifted by sigma = (T - cnt) mod 4
+  const long long c0 = desc ? t0 + ((T - cnt) & 3) + cnt - T : t0;
   store_tile<E, U, PAIRS>(sk, sv, key, val, tid * E, cnt, desc, args.out_k, args.out_v, c0,
                           args.decode_f32 != 0);
 }

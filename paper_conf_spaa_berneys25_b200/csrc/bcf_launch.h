@@ -16,6 +16,7 @@ struct Variant {
   BlockSortFn block_sort = nullptr;
   MergeFn merge = nullptr;        // regular pass (CF: B runs stored descending)
   MergeFn merge_table = nullptr;  // group-table pass, all runs ascending (CF)
+  MergeFn merge_tma = nullptr;    // persistent TMA pass (CF, E coprime with 32); grid arg = tiles
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]

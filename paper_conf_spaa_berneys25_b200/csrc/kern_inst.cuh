@@ -2,6 +2,7 @@
 // three block sizes; included by kern_E<E>.cu with BCF_E defined.
 #pragma once
 #include "bcf_kernels.cuh"
+#include "bcf_merge_tma.cuh"
 #include "bcf_launch.h"
 
 namespace bcf {
@@ -37,6 +38,39 @@ cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+// persistent TMA merge pass: grid = min(tiles, SMs x resident CTAs), each
+// CTA a contiguous chunk of tiles
+template <int E, int U, bool PAIRS>
+cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s) {
+  constexpr size_t smem = tma_smem_bytes<E, U, PAIRS>();
+  auto kern = merge_pass_tma_kernel<E, U, PAIRS>;
+  static int per_sm[32] = {0};
+  static int nsm[32] = {0};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev >= 32) return cudaErrorInvalidDevice;
+  if (per_sm[dev] == 0) {
+    if (smem > 48 * 1024) {
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e != cudaSuccess) return e;
+    }
+    int k = 0, sms = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, U + 32, smem);
+    if (e != cudaSuccess) return e;
+    e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess) return e;
+    nsm[dev] = sms;
+    per_sm[dev] = k > 0 ? k : 1;
+  }
+  long long ctas = (long long)nsm[dev] * per_sm[dev];
+  if (ctas > tiles) ctas = tiles;
+  const long long per_cta = (tiles + ctas - 1) / ctas;
+  ctas = (tiles + per_cta - 1) / per_cta;
+  kern<<<(unsigned)ctas, U + 32, smem, s>>>(a, tiles, per_cta);
+  return cudaGetLastError();
+}
+
 template <int E, int U>
 void register_eu(LaunchTable& t) {
   const int ui = u_index(U);
@@ -46,6 +80,10 @@ void register_eu(LaunchTable& t) {
                       &launch_merge<E, U, true, true, false>};
   t.v[E][ui][1][0] = {&launch_block_sort<E, U, false, false>, &launch_merge<E, U, false, false, false>,
                       nullptr};
+  if constexpr (cgcd(W, E) == 1) {
+    t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
+    t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;
+  }
 }
 
 }  // namespace bcf
