@@ -141,6 +141,9 @@ bcf_status bcf_profile_enable(int32_t on);
 bcf_status bcf_profile_collect(bcf_kernel_stats* out, int32_t max, int32_t* count);
 /* total kernels launched by this process through the library (always on) */
 int64_t bcf_launch_count(void);
+/* debug: copy the per-CTA timeline recorded for merge pass $BCF_TRACE (globaltimer
+   ns; 256 slots per CTA) into host memory; BCF_ERROR_INVALID_VALUE if none */
+bcf_status bcf_debug_trace_copy(void* host, uint64_t bytes);
 
 #ifdef __cplusplus
 }

@@ -20,7 +20,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbcf.so")
+LIB_PATH = os.environ.get("BCF_LIB") or os.path.join(_HERE, "libbcf.so")  # BCF_LIB: A/B builds
 
 BCF_SUCCESS = 0
 BCF_ERROR_INVALID_VALUE = 1
@@ -35,7 +35,7 @@ EXPORTED_SYMBOLS = [
     "bcf_default_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
     "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
-    "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count",
+    "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
 ]
 
 

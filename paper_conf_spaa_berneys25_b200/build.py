@@ -53,7 +53,23 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None,
+          defines=(), lib: str | None = None, obj: str | None = None) -> str:
+    """defines/lib/obj: extra -D flags and output paths for A/B variant builds."""
+    global OBJ, LIB, NVCC_FLAGS
+    saved = (OBJ, LIB, NVCC_FLAGS)
+    if obj:
+        OBJ = obj
+    if lib:
+        LIB = lib
+    NVCC_FLAGS = NVCC_FLAGS + ["-D" + d for d in defines]
+    try:
+        return _build(force, verbose, jobs)
+    finally:
+        OBJ, LIB, NVCC_FLAGS = saved
+
+
+def _build(force, verbose, jobs):
     os.makedirs(OBJ, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
     if force:

@@ -114,6 +114,22 @@ static bcf_status resolve(const bcf_params* p, Params& out) {
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+// BCF_TRACE=<pass>: record a per-CTA timeline of that merge pass (debug)
+static unsigned long long* g_trace = nullptr;
+static const size_t TRACE_WORDS = 1 << 21;
+static unsigned long long* trace_for_pass(int pass) {
+  static const int want = [] {
+    const char* v = getenv("BCF_TRACE");
+    return v ? atoi(v) : -1;
+  }();
+  if (pass != want) return nullptr;
+  if (!g_trace) {
+    if (cudaMalloc(&g_trace, TRACE_WORDS * 8) != cudaSuccess) return nullptr;
+    cudaMemset(g_trace, 0, TRACE_WORDS * 8);
+  }
+  return g_trace;
+}
+
 // BCF_NO_TMA=1 selects the non-persistent merge kernel (A/B measurements)
 static bool tma_disabled() {
   static const bool off = [] {
@@ -176,7 +192,7 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
     uint32_t* dk = i == P ? out_k : ((i & 1) ? Y : X);
     uint32_t* dv = i == P ? out_v : ((i & 1) ? YV : XV);
     MergeArgs ma{sk, sv, dk, dv, (long long)n, T << (i - 1), i,
-                 (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0};
+                 (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0, trace_for_pass(i)};
     if (use_tma)
       e = launch("merge_pass", n, s, [&] { return var.merge_tma(ma, tiles, s); });
     else
@@ -350,7 +366,7 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     GroupDesc* dt = dtab + (size_t)(i - 1) * (table_bytes / sizeof(GroupDesc));
     cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_fail(e);
-    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, 0, dt, (int)tab.size()};
+    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
     e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
     if (e != cudaSuccess) return cuda_fail(e);
     srck = bk[dst];
@@ -408,5 +424,12 @@ bcf_status bcf_profile_collect(bcf_kernel_stats* out, int32_t max, int32_t* coun
 }
 
 int64_t bcf_launch_count(void) { return g_launches.load(); }
+
+bcf_status bcf_debug_trace_copy(void* host, uint64_t bytes) {
+  if (!g_trace) return BCF_ERROR_INVALID_VALUE;
+  if (bytes > TRACE_WORDS * 8) bytes = TRACE_WORDS * 8;
+  cudaError_t e = cudaMemcpy(host, g_trace, bytes, cudaMemcpyDeviceToHost);
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
 
 }  // extern "C"

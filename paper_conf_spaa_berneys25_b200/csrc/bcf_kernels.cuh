@@ -64,6 +64,7 @@ struct MergeArgs {
   int cf_dirs;     // regular mode: odd runs descending
   const GroupDesc* groups;  // table mode (merge of arbitrary runs) if non-null
   int ngroups;
+  unsigned long long* trace;  // debug timeline (BCF_TRACE), nullptr normally
 };
 
 // Group of output tile `tile`: regular pairwise pass (run 2g with run 2g+1,

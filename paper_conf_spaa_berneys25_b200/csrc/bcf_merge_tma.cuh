@@ -30,7 +30,18 @@
 
 namespace bcf {
 
-constexpr int TMA_STAGES = 2;
+#ifndef BCF_TMA_STAGES
+#define BCF_TMA_STAGES 3
+#endif
+#ifndef BCF_TMA_MINB
+#define BCF_TMA_MINB 1
+#endif
+// startup boundary search: 0 = producer only (sequential), 1 = every warp,
+// 64-ary; 2 = every warp, 32-ary
+#ifndef BCF_STARTUP
+#define BCF_STARTUP 1
+#endif
+constexpr int TMA_STAGES = BCF_TMA_STAGES;
 
 template <int E, int U>
 __host__ __device__ constexpr int stage_words() {
@@ -46,10 +57,24 @@ struct TileMeta {
   int NA, NB, cnt, c, cout, qlo, qhi, desc;
 };
 
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+// debug timeline: 256 slots per CTA (consumers at 1 + 4i, producer at 128 + 4i)
+#define BCF_TRACE_AT(slot)                                                          \
+  do {                                                                              \
+    if (args.trace && (slot) < 256) args.trace[(size_t)blockIdx.x * 256 + (slot)] = gtimer(); \
+  } while (0)
+
 __device__ __forceinline__ int align_up4(int x) { return (x + 3) & ~3; }
 __device__ __forceinline__ int align_dn4(int x) { return x & ~3; }
 
-// merge path with an initial bracket [lo, hi] (all lanes get the answer)
+// merge path with an initial bracket [lo, hi] (all lanes get the answer):
+// 64-ary search, every lane tests two candidates per round (4 independent
+// loads in flight), so a bracket of one tile (<= 4096) takes 2 rounds of
+// global-memory latency and a full run of 2^23 takes 4.
 __device__ __forceinline__ long long merge_path_warp_global_bounded(const RunView& A, const RunView& B,
                                                                     long long D, long long lo, long long hi,
                                                                     int lane) {
@@ -60,15 +85,15 @@ __device__ __forceinline__ long long merge_path_warp_global_bounded(const RunVie
   if (hi > h2) hi = h2;
   while (hi > lo) {
     const long long cnt = hi - lo;
-    const long long s = (cnt + 31) >> 5;
-    const long long m = lo + (long long)(lane + 1) * s - 1;
-    bool p = false;
-    if (m < hi) {
-      const uint32_t a = A.ld(m);
-      const uint32_t b = B.ld(D - 1 - m);
-      p = !(b < a);
-    }
-    const int c = __popc(__ballot_sync(FULL, p));
+    const long long s = (cnt + 63) >> 6;  // probe stride, 64 probes
+    const long long m0 = lo + (long long)(2 * lane + 1) * s - 1;
+    const long long m1 = m0 + s;
+    uint32_t a0 = 0, b0 = 0, a1 = 0, b1 = 0;
+    if (m0 < hi) { a0 = A.ld(m0); b0 = B.ld(D - 1 - m0); }
+    if (m1 < hi) { a1 = A.ld(m1); b1 = B.ld(D - 1 - m1); }
+    const bool p0 = m0 < hi && !(b0 < a0);
+    const bool p1 = m1 < hi && !(b1 < a1);
+    const int c = __popc(__ballot_sync(FULL, p0)) + __popc(__ballot_sync(FULL, p1));
     const long long nlo = lo + (long long)c * s;
     long long nhi = lo + (long long)(c + 1) * s - 1;
     if (nhi > hi) nhi = hi;
@@ -78,8 +103,38 @@ __device__ __forceinline__ long long merge_path_warp_global_bounded(const RunVie
   return lo;
 }
 
+// Bracketed merge path that first tests the 64 candidates around a guess
+// (the proportional split of the remaining elements): for random keys the
+// answer lies within +-32 of it with high probability (one round of global
+// latency); otherwise the 64-ary search continues on the reduced bracket.
+__device__ __forceinline__ long long merge_path_warp_global_guess(const RunView& A, const RunView& B,
+                                                                  long long D, long long lo, long long hi,
+                                                                  long long guess, int lane) {
+  long long l2 = D - B.len;
+  if (lo < l2) lo = l2;
+  if (lo < 0) lo = 0;
+  long long h2 = D < A.len ? D : A.len;
+  if (hi > h2) hi = h2;
+  if (hi <= lo) return lo;
+  long long L = guess - 32;
+  if (L > hi - 64) L = hi - 64;
+  if (L < lo) L = lo;
+  const long long m0 = L + 2 * lane, m1 = m0 + 1;
+  uint32_t a0 = 0, b0 = 0, a1 = 0, b1 = 0;
+  if (m0 < hi) { a0 = A.ld(m0); b0 = B.ld(D - 1 - m0); }
+  if (m1 < hi) { a1 = A.ld(m1); b1 = B.ld(D - 1 - m1); }
+  const bool p0 = m0 < hi && !(b0 < a0);
+  const bool p1 = m1 < hi && !(b1 < a1);
+  const int c = __popc(__ballot_sync(FULL, p0)) + __popc(__ballot_sync(FULL, p1));
+  long long act = hi - L;
+  if (act > 64) act = 64;
+  if (c > 0 && c < act) return L + c;                 // exact: Q(L+c-1) true, Q(L+c) false
+  if (c == 0) return L == lo ? lo : merge_path_warp_global_bounded(A, B, D, lo, L, lane);
+  return L + c == hi ? hi : merge_path_warp_global_bounded(A, B, D, L + c, hi, lane);
+}
+
 template <int E, int U, bool PAIRS>
-__global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, long long tiles,
+__global__ void __launch_bounds__(U + 32, BCF_TMA_MINB) merge_pass_tma_kernel(MergeArgs args, long long tiles,
                                                                 long long per_cta) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
@@ -91,6 +146,7 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
   __shared__ __align__(8) uint64_t full_bar[S];
   __shared__ __align__(8) uint64_t empty_bar[S];
   __shared__ int s_org[NW + 1];
+  __shared__ long long s_bnd[NW + 2];  // precomputed boundaries (see below)
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
@@ -108,6 +164,32 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
     for (int s = 0; s < S; ++s) {
       tma::mbar_init(&full_bar[s], 1);
       tma::mbar_init(&empty_bar[s], 1);
+    }
+  }
+  // Startup: the NW + 1 warps compute, in parallel, the merge-path
+  // boundaries of the first tiles of the chunk (full-range 64-ary searches):
+  // s_bnd[k] = a(start of tile k) for k < min(m, NW + 1), and
+  // s_bnd[NW + 1] = a(end of the last tile) when m <= NW + 1.  The producer's
+  // steady state then starts with no search on its critical path.
+  const int npre = BCF_STARTUP == 0 ? 0 : (m < NW + 1 ? m : NW + 1);
+  if (BCF_STARTUP != 0) {
+    int k = warp;
+    const bool last = (m <= NW + 1) && (warp == m % (NW + 1));  // spare warp: end of last tile
+    if (k < npre || last) {
+      const long long t = t_begin + (last ? m - 1 : k);
+      long long j;
+      const GroupDesc grp = group_of_tile(args, t, T, j);
+      const long long lenG = grp.na + grp.nb;
+      long long D = j * T;
+      if (last) D = D + T < lenG ? D + T : lenG;
+      RunView Av{args.src_k + grp.a_off, grp.na, 0};
+      RunView Bv{args.src_k + grp.b_off, grp.nb, 1};
+      long long a;
+      if (D == 0) a = 0;
+      else if (D == lenG) a = grp.na;
+      else if (BCF_STARTUP == 2) a = merge_path_warp_global(Av, Bv, D, lane);
+      else a = merge_path_warp_global_bounded(Av, Bv, D, 0, D, lane);
+      if (lane == 0) s_bnd[last ? NW + 1 : k] = a;
     }
   }
   __syncthreads();
@@ -130,10 +212,12 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
       const long long g0 = M.c0 - M.cout;                  // global word of stage word 0
       int ilo = align_up4(w0), ihi = align_dn4(w1);
       if (ihi <= ilo) ilo = ihi = w1;  // tiny tile: everything via lanes
-      if (lane == 0 && ihi > ilo) {
-        tma::bulk_s2g(dstk + g0 + ilo, sk + ilo, (uint32_t)(ihi - ilo) * 4u);
-        if constexpr (PAIRS) tma::bulk_s2g(dstv + g0 + ilo, sv + ilo, (uint32_t)(ihi - ilo) * 4u);
-        tma::bulk_commit();
+      if (lane == 0) {
+        if (ihi > ilo) {
+          tma::bulk_s2g(dstk + g0 + ilo, sk + ilo, (uint32_t)(ihi - ilo) * 4u);
+          if constexpr (PAIRS) tma::bulk_s2g(dstv + g0 + ilo, sv + ilo, (uint32_t)(ihi - ilo) * 4u);
+        }
+        tma::bulk_commit();  // one group per tile (possibly empty): wait_group counts tiles
       }
       // head words [w0, ilo) and tail words [ihi, w1): at most 3 + 3 (or 7)
       {
@@ -146,14 +230,20 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
           if constexpr (PAIRS) dstv[g0 + w] = sv[w];
         }
       }
-      if (lane == 0) tma::bulk_wait_read_all();
       __syncwarp();
     };
 
-    for (int i = 0; i < m; ++i) {
-      const int s = i % S;
-      const uint32_t u = (uint32_t)(i / S);
-      const long long t = t_begin + i;
+    // Split of tile t (merge-path boundaries a0, a1 and the tile descriptor);
+    // consecutive tiles of the chunk reuse the previous boundary, so the
+    // search for a1 is bracketed to a range of T (3 rounds of 32 probes).
+    struct Split {
+      TileMeta M;
+      long long oA, oB;
+      int ea0, ea1, eb0, eb1, a_hi, b_lo, b_hi;  // copy plan (stage words)
+      int ew;                                    // this lane's edge word (-1: none)
+      uint32_t ek, ev;                           // its value (loaded early)
+    };
+    auto split_of = [&](long long t) {
       long long j;
       const GroupDesc grp = group_of_tile(args, t, T, j);
       const long long lenG = grp.na + grp.nb;
@@ -161,91 +251,144 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
       const long long D1 = D0 + T < lenG ? D0 + T : lenG;
       RunView Av{srck + grp.a_off, grp.na, 0};
       RunView Bv{srck + grp.b_off, grp.nb, 1};
+      const int i = (int)(t - t_begin);
       long long a0;
-      if (j == 0) a0 = 0;
+      if (i < npre) a0 = s_bnd[i];
+      else if (j == 0) a0 = 0;
       else if (prev_tb == grp.tile_begin) a0 = prev_a1;  // consecutive tile, same group
-      else a0 = merge_path_warp_global(Av, Bv, D0, lane);
+      else a0 = merge_path_warp_global_bounded(Av, Bv, D0, 0, D0, lane);
       long long a1;
       if (D1 == lenG) a1 = grp.na;
-      else a1 = merge_path_warp_global_bounded(Av, Bv, D1, a0, a0 + (D1 - D0), lane);
+      else if (i + 1 < npre) a1 = s_bnd[i + 1];
+      else if (npre > 0 && i + 1 == m && m <= NW + 1) a1 = s_bnd[NW + 1];
+      else {
+        const long long rest = lenG - D0;
+        const long long guess = a0 + (long long)((double)(D1 - D0) * (double)(grp.na - a0) / (double)rest);
+        a1 = merge_path_warp_global_guess(Av, Bv, D1, a0, a0 + (D1 - D0), guess, lane);
+      }
       prev_a1 = a1;
       prev_tb = grp.tile_begin;
+      // L2 prefetch of the next tile's A and B ranges: they hold the probes
+      // of the next split search and the next bulk loads
+      if (lane == 0 && D1 < lenG) {
+        const long long b1 = D1 - a1;
+        const long long ahi = a1 + T < grp.na ? a1 + T : grp.na;
+        const long long bhi = b1 + T < grp.nb ? b1 + T : grp.nb;
+        if (ahi > a1) {
+          const long long w0 = (grp.a_off + a1) & ~3ll, w1 = (grp.a_off + ahi + 3) & ~3ll;
+          tma::bulk_prefetch_l2(srck + w0, (uint32_t)(w1 - w0) * 4u);
+        }
+        if (bhi > b1) {  // B[y] at b_off + nb-1-y: y in [b1, bhi) -> [b_off+nb-bhi, b_off+nb-b1)
+          const long long w0 = (grp.b_off + grp.nb - bhi) & ~3ll, w1 = (grp.b_off + grp.nb - b1 + 3) & ~3ll;
+          tma::bulk_prefetch_l2(srck + w0, (uint32_t)(w1 - w0) * 4u);
+        }
+      }
+      Split sp;
       const int cnt = (int)(D1 - D0);
-      const int NA = (int)(a1 - a0);
-      const int NB = cnt - NA;
       const long long b0 = D0 - a0;
-      const long long oA = grp.a_off + a0;                     // A[a0 + q] at word oA + q
-      const long long oB = grp.b_off + grp.nb - b0 - T;        // logical q (B part) at oB + q
-      const int c = (int)(oA & 3);                             // src is 16-byte aligned
-      TileMeta M;
-      M.desc = grp.out_desc;
-      M.c0 = M.desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
-      M.qlo = M.desc ? T - cnt : 0;
-      M.qhi = M.desc ? T : cnt;
-      M.cout = (int)((unsigned long long)(dst_phase + M.c0) & 3ull);
-      M.NA = NA;
-      M.NB = NB;
-      M.cnt = cnt;
-      M.c = c;
-
-      if (i >= S) {
-        tma::mbar_wait(&empty_bar[s], (u - 1) & 1);
-        store_out(s);
+      sp.oA = grp.a_off + a0;                     // A[a0 + q] at word oA + q
+      sp.oB = grp.b_off + grp.nb - b0 - T;        // logical q (B part) at oB + q
+      sp.M.desc = grp.out_desc;
+      sp.M.c0 = sp.M.desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
+      sp.M.qlo = sp.M.desc ? T - cnt : 0;
+      sp.M.qhi = sp.M.desc ? T : cnt;
+      sp.M.cout = (int)((unsigned long long)(dst_phase + sp.M.c0) & 3ull);
+      const int NA = (int)(a1 - a0), NB = cnt - NA, c = (int)(sp.oA & 3);  // src 16-B aligned
+      sp.M.NA = NA;
+      sp.M.NB = NB;
+      sp.M.cnt = cnt;
+      sp.M.c = c;
+      // copy plan: logical q lives at stage word c + q; A -> [0, a_hi),
+      // B -> [b_lo, b_hi); a 16-byte chunk shared by A's tail and B's head is
+      // filled word by word (edge words)
+      sp.a_hi = NA ? align_up4(c + NA) : 0;
+      sp.b_lo = NB ? align_dn4(c + T - NB) : 0;
+      sp.b_hi = NB ? align_up4(c + T) : 0;
+      sp.ea0 = sp.ea1 = sp.eb0 = sp.eb1 = 0;
+      if (NA && NB && sp.a_hi > sp.b_lo) {
+        sp.ea1 = c + NA;
+        sp.a_hi = align_dn4(sp.ea1);
+        sp.ea0 = sp.a_hi;
+        sp.eb0 = c + T - NB;
+        sp.b_lo = align_up4(sp.eb0);
+        sp.eb1 = sp.b_lo;
       }
-      if (lane == 0) meta[s] = M;
-
-      // copy ranges in stage words: logical q lives at stage word c + q
-      int a_hi = NA ? align_up4(c + NA) : 0;           // A: stage [0, a_hi)
-      int b_lo = NB ? align_dn4(c + T - NB) : 0;       // B: stage [b_lo, b_hi)
-      const int b_hi = NB ? align_up4(c + T) : 0;
-      int ea0 = 0, ea1 = 0, eb0 = 0, eb1 = 0;          // edge words (stage indices)
-      if (NA && NB && a_hi > b_lo) {
-        ea1 = c + NA;
-        a_hi = align_dn4(ea1);
-        ea0 = a_hi;
-        eb0 = c + T - NB;
-        b_lo = align_up4(eb0);
-        eb1 = b_lo;
+      // issue the edge-word loads now; they are consumed by load_tile later
+      sp.ew = -1;
+      sp.ek = sp.ev = 0;
+      long long gw = 0;
+      if (lane >= 1 && lane <= 3 && sp.ea0 + lane - 1 < sp.ea1) {
+        sp.ew = sp.ea0 + lane - 1;
+        gw = sp.oA + (sp.ew - c);
+      } else if (lane >= 4 && lane <= 6 && sp.eb0 + lane - 4 < sp.eb1) {
+        sp.ew = sp.eb0 + lane - 4;
+        gw = sp.oB + (sp.ew - c);
       }
+      if (sp.ew >= 0) {
+        sp.ek = __ldg(srck + gw);
+        if constexpr (PAIRS) sp.ev = __ldg(srcv + gw);
+      }
+      return sp;
+    };
+
+    // bulk loads of tile i (described by sp) into stage s
+    auto load_tile = [&](int s, const Split& sp) {
+      if (lane == 0) meta[s] = sp.M;
       uint32_t* sk = stage_k(s);
       uint32_t* sv = stage_v(s);
+      const int c = sp.M.c;
       if (lane == 0) {
-        const uint32_t bytes = (uint32_t)(a_hi + (b_hi - b_lo)) * 4u * (PAIRS ? 2u : 1u);
+        const uint32_t bytes = (uint32_t)(sp.a_hi + (sp.b_hi - sp.b_lo)) * 4u * (PAIRS ? 2u : 1u);
         tma::mbar_expect_tx(&full_bar[s], bytes);
-        if (a_hi > 0) {
-          tma::bulk_g2s(sk, srck + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
-          if constexpr (PAIRS) tma::bulk_g2s(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
+        if (sp.a_hi > 0) {
+          tma::bulk_g2s(sk, srck + (sp.oA - c), (uint32_t)sp.a_hi * 4u, &full_bar[s]);
+          if constexpr (PAIRS) tma::bulk_g2s(sv, srcv + (sp.oA - c), (uint32_t)sp.a_hi * 4u, &full_bar[s]);
         }
-        if (b_hi > b_lo) {
-          tma::bulk_g2s(sk + b_lo, srck + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
-          if constexpr (PAIRS)
-            tma::bulk_g2s(sv + b_lo, srcv + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        if (sp.b_hi > sp.b_lo) {
+          const uint32_t nb = (uint32_t)(sp.b_hi - sp.b_lo) * 4u;
+          tma::bulk_g2s(sk + sp.b_lo, srck + (sp.oB + sp.b_lo - c), nb, &full_bar[s]);
+          if constexpr (PAIRS) tma::bulk_g2s(sv + sp.b_lo, srcv + (sp.oB + sp.b_lo - c), nb, &full_bar[s]);
         }
       }
-      // misaligned edge words around the A/B boundary (generic loads/stores)
-      {
-        int w = -1;
-        long long gw = 0;
-        if (lane >= 1 && lane <= 3 && ea0 + lane - 1 < ea1) {
-          w = ea0 + lane - 1;
-          gw = oA + (w - c);
-        } else if (lane >= 4 && lane <= 6 && eb0 + lane - 4 < eb1) {
-          w = eb0 + lane - 4;
-          gw = oB + (w - c);
-        }
-        if (w >= 0) {
-          sk[w] = __ldg(srck + gw);
-          if constexpr (PAIRS) sv[w] = __ldg(srcv + gw);
-        }
+      if (sp.ew >= 0) {
+        sk[sp.ew] = sp.ek;
+        if constexpr (PAIRS) sv[sp.ew] = sp.ev;
       }
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);
-    }
-    // drain: store the last min(S, m) tiles
-    for (int i = (m > S ? m - S : 0); i < m; ++i) {
+    };
+
+    // Schedule per tile i (S = 3 stages):
+    //   wait for tile i-2's outputs, issue its bulk store (no read wait);
+    //   wait until tile i-3's store has read its stage (issued one step ago);
+    //   load tile i into that stage; search the split of tile i+1 while the
+    //   consumers compute tile i-1.
+    if (lane == 0) BCF_TRACE_AT(0);
+    if (lane == 0) BCF_TRACE_AT(128);
+    Split cur = split_of(t_begin);
+    if (lane == 0) BCF_TRACE_AT(129);
+    for (int i = 0; i < m; ++i) {
       const int s = i % S;
-      tma::mbar_wait(&empty_bar[s], (uint32_t)(i / S) & 1);
-      store_out(s);
+      if (i >= 2) {
+        const int k = i - 2;
+        tma::mbar_wait(&empty_bar[k % S], (uint32_t)(k / S) & 1);
+        if (lane == 0) BCF_TRACE_AT(128 + 4 * i + 3);
+        store_out(k % S);  // issue + commit, no read wait
+      }
+      if (i >= S) {
+        // stage s held tile i-3, whose store was committed one step ago
+        if (lane == 0) tma::bulk_wait_read_1();
+        __syncwarp();
+      }
+      load_tile(s, cur);
+      if (lane == 0) BCF_TRACE_AT(128 + 4 * i + 2);
+      if (i + 1 < m) cur = split_of(t_begin + i + 1);
+      if (lane == 0) BCF_TRACE_AT(128 + 4 * (i + 1) + 1);
+    }
+    // drain: the last two tiles
+    for (int k = (m >= 2 ? m - 2 : 0); k < m; ++k) {
+      tma::mbar_wait(&empty_bar[k % S], (uint32_t)(k / S) & 1);
+      store_out(k % S);
     }
     if (lane == 0) tma::bulk_wait_all();
     return;
@@ -255,7 +398,9 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
   const bool decode = args.decode_f32 != 0;
   for (int i = 0; i < m; ++i) {
     const int s = i % S;
+    if (tid == 0) BCF_TRACE_AT(1 + 4 * i);
     tma::mbar_wait(&full_bar[s], (uint32_t)(i / S) & 1);
+    if (tid == 0) BCF_TRACE_AT(2 + 4 * i);
     const TileMeta M = meta[s];
     uint32_t* sk = stage_k(s) + M.c;  // logical index -> sk[index]
     uint32_t* sv = stage_v(s) + M.c;
@@ -303,6 +448,7 @@ __global__ void __launch_bounds__(U + 32) merge_pass_tma_kernel(MergeArgs args, 
     tma::fence_proxy_async_smem();
     tma::named_bar_sync(1, U);
     if (tid == 0) tma::mbar_arrive(&empty_bar[s]);
+    if (tid == 0) BCF_TRACE_AT(3 + 4 * i);
   }
 }
 

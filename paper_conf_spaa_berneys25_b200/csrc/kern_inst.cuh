@@ -3,6 +3,7 @@
 #pragma once
 #include "bcf_kernels.cuh"
 #include "bcf_merge_tma.cuh"
+#include "bcf_merge_win.cuh"
 #include "bcf_launch.h"
 
 namespace bcf {
@@ -40,35 +41,51 @@ cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
 
 // persistent TMA merge pass: grid = min(tiles, SMs x resident CTAs), each
 // CTA a contiguous chunk of tiles
-template <int E, int U, bool PAIRS>
-cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s) {
-  constexpr size_t smem = tma_smem_bytes<E, U, PAIRS>();
-  auto kern = merge_pass_tma_kernel<E, U, PAIRS>;
-  static int per_sm[32] = {0};
-  static int nsm[32] = {0};
+struct PersistentCache {
+  int per_sm[32] = {0};
+  int nsm[32] = {0};
+};
+
+template <typename K>
+cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int threads, const MergeArgs& a,
+                              long long tiles, cudaStream_t s) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (dev >= 32) return cudaErrorInvalidDevice;
-  if (per_sm[dev] == 0) {
+  if (pc.per_sm[dev] == 0) {
     if (smem > 48 * 1024) {
       e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       if (e != cudaSuccess) return e;
     }
     int k = 0, sms = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, U + 32, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, threads, smem);
     if (e != cudaSuccess) return e;
     e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     if (e != cudaSuccess) return e;
-    nsm[dev] = sms;
-    per_sm[dev] = k > 0 ? k : 1;
+    pc.nsm[dev] = sms;
+    pc.per_sm[dev] = k > 0 ? k : 1;
   }
-  long long ctas = (long long)nsm[dev] * per_sm[dev];
+  long long ctas = (long long)pc.nsm[dev] * pc.per_sm[dev];
   if (ctas > tiles) ctas = tiles;
   const long long per_cta = (tiles + ctas - 1) / ctas;
   ctas = (tiles + per_cta - 1) / per_cta;
-  kern<<<(unsigned)ctas, U + 32, smem, s>>>(a, tiles, per_cta);
+  kern<<<(unsigned)ctas, threads, smem, s>>>(a, tiles, per_cta);
   return cudaGetLastError();
+}
+
+#ifndef BCF_MERGE_WIN
+#define BCF_MERGE_WIN 1
+#endif
+template <int E, int U, bool PAIRS>
+cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s) {
+  static PersistentCache pc;  // one per (E, U, PAIRS) instantiation
+  if constexpr (!PAIRS && BCF_MERGE_WIN) {
+    return launch_persistent(merge_pass_win_kernel<E, U>, pc, win_smem_bytes<E, U>(), U + 32, a, tiles, s);
+  } else {
+    return launch_persistent(merge_pass_tma_kernel<E, U, PAIRS>, pc, tma_smem_bytes<E, U, PAIRS>(), U + 32,
+                             a, tiles, s);
+  }
 }
 
 template <int E, int U>
@@ -88,11 +105,25 @@ void register_eu(LaunchTable& t) {
 
 }  // namespace bcf
 
+// BCF_ONLY_E / BCF_ONLY_U (A/B experiment builds): instantiate one (E, u)
+#ifndef BCF_ONLY_U
+#define BCF_REG_U(E, U) register_eu<E, U>(t);
+#else
+#define BCF_REG_U(E, U) \
+  if constexpr (U == BCF_ONLY_U) register_eu<E, U>(t);
+#endif
 #define BCF_DEFINE_REG(E)                         \
   namespace bcf {                                 \
   void register_E##E(LaunchTable& t) {            \
-    register_eu<E, 128>(t);                       \
-    register_eu<E, 256>(t);                       \
-    register_eu<E, 512>(t);                       \
+    if constexpr (BCF_E_ENABLED(E)) {             \
+      BCF_REG_U(E, 128)                           \
+      BCF_REG_U(E, 256)                           \
+      BCF_REG_U(E, 512)                           \
+    }                                             \
   }                                               \
   }
+#ifdef BCF_ONLY_E
+#define BCF_E_ENABLED(E) ((E) == BCF_ONLY_E)
+#else
+#define BCF_E_ENABLED(E) true
+#endif
