@@ -220,48 +220,48 @@ __device__ __forceinline__ int lane_split_smem(const uint32_t* __restrict__ sk, 
   const int ib = beta + lp * E;
   const uint32_t cA = ia < NA ? lds<E>(sk, base + ia) : 0u;
   const uint32_t cB = ib < NB ? lds<E>(sk, base + S2 - 1 - ib) : 0u;
-  // coarse cell: largest m in [0, lp] with Q(alpha + mE), bisection over lanes
-  int lo = 0, hi = lp + 1;  // Q(lo) true, answer < hi
-  for (int it = 0; it < nit; ++it) {
-    const int mid = (lo + hi) >> 1;
-    const bool live = hi - lo > 1;
-    const int m = live ? mid : lo;
-    const uint32_t a = __shfl_sync(FULL, cA, wb + (m >= 1 ? m - 1 : 0));
-    const uint32_t b = __shfl_sync(FULL, cB, wb + lp - m);
-    const bool validA = alpha + m * E <= NA;
-    const bool validB = beta + (lp - m) * E < NB;
-    const bool q = (m == 0) || (validA && (!validB || !(b < a)));
-    if (live) {
-      lo = q ? m : lo;
-      hi = q ? hi : m;
+  // coarse cell: largest m in [0, lp] with Q(alpha + mE), built bit by bit
+  // (lanes of the window hold the corners; two shuffles per step).
+  //   Q(m) = A-corner m-1 exists (m <= mA) and (B-corner lp-m is past B's end
+  //          (lp - m >= kB) or !(B corner < A corner))
+  const int mA = (NA - alpha) / E;
+  const int kB = NB - beta > 0 ? (NB - beta + E - 1) / E : 0;
+  int M = 0;
+#pragma unroll
+  for (int it = 0; it < 5; ++it) {
+    const int st = 16 >> it;
+    if (st < WL) {  // warp-uniform
+      const int cnd = M + st;
+      const bool inr = cnd <= lp;
+      const uint32_t a = __shfl_sync(FULL, cA, wb + (inr ? cnd - 1 : 0));
+      const uint32_t b = __shfl_sync(FULL, cB, wb + (inr ? lp - cnd : 0));
+      const bool q = inr && cnd <= mA && (lp - cnd >= kB || !(b < a));
+      M = q ? cnd : M;
     }
   }
+  (void)nit;
   // (3) cell scan: round j tests Q(ac + j + 1) reading A[ac+j] and B[D-ac-1-j]
-  const int ac = alpha + lo * E;  // a(D) in [ac, ac+E]
+  const int ac = alpha + M * E;  // a(D) in [ac, ac+E]
   const int jA = (NA < D ? NA : D) - ac;   // j < jA: A[ac+j] exists and ac+j+1 <= D
   const int jB = D - ac - NB;              // j >= jB: B[D-ac-1-j] exists
   const int pa0 = base + ac;               // logical index of A[ac + j] = pa0 + j
   const int pb0 = base + S2 - D + ac;      // logical index of B[D-ac-1-j] = pb0 + j
-  // Probes outside [jB, jA) are still issued (their logical indices stay in
-  // the same round set, so they cannot conflict; the tile buffer has E words
-  // of slack past its end) and masked out of the count.
-  int cnt = 0;
-  if (__all_sync(FULL, jA >= E && jB <= 0)) {
-    // interior of the tile (all lanes): no masking needed
+  // Every probe is issued (indices outside [jB, jA) stay in the same round set,
+  // so they cannot conflict; the tile buffer has E words of slack past its
+  // end); the comparison bits are collected in a mask and the predicate is
+  // true below jB, monotone on [jB, jA), false from jA on.
+  uint32_t tm = 0;
 #pragma unroll
-    for (int j = 0; j < E; ++j) {
-      const uint32_t ka = lds<E>(sk, pa0 + j);
-      const uint32_t kb = lds<E>(sk, pb0 + j);
-      cnt += (kb < ka) ? 0 : 1;
-    }
-  } else {
-#pragma unroll
-    for (int j = 0; j < E; ++j) {
-      const uint32_t ka = lds<E>(sk, pa0 + j);
-      const uint32_t kb = lds<E>(sk, pb0 + j);
-      cnt += (j < jA && (j < jB || !(kb < ka))) ? 1 : 0;
-    }
+  for (int j = 0; j < E; ++j) {
+    const uint32_t ka = lds<E>(sk, pa0 + j);
+    const uint32_t kb = lds<E>(sk, pb0 + j);
+    tm |= (kb < ka) ? 0u : (1u << j);
   }
+  // (past the end of the merge, D > NA + NB, jB exceeds jA: clamp)
+  const int jAc = jA < 0 ? 0 : (jA > E ? E : jA);
+  const int jBc = jB < 0 ? 0 : (jB > jAc ? jAc : jB);
+  const uint32_t range = ((1u << jAc) - 1u) & ~((1u << jBc) - 1u);
+  const int cnt = jBc + __popc(tm & range);
   return ac + cnt;
 }
 
@@ -281,15 +281,18 @@ __device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restri
                                                         uint32_t pad) {
   const int k = a % E;
   // round j: ia = (j - k) mod E; A_i[ia] at logical base+a+ia, else
-  // B_i[E-1-ia] at base+S2-1-(b+E-1-ia) = base+S2-b-E+ia
+  // B_i[E-1-ia] at base+S2-1-(b+E-1-ia) = base+S2-b-E+ia.  Rounds reading A
+  // form the circular range [k, k+nA): bit j of maskA.
   const int offA = base + a - k;
   const int offB = base + S2 - b - E - k;
-  const int hiA = k + nA;  // A rounds: j in [k, k+nA) (mod E)
+  const uint32_t m0 = (1u << nA) - 1u;
+  const uint32_t maskA = ((m0 << k) | (m0 >> (E - k))) & ((1u << E) - 1u);
+  const int bAn = offA, bAw = offA + E, bBn = offB, bBw = offB + E;
 #pragma unroll
   for (int j = 0; j < E; ++j) {
     const bool wrap = j < k;
-    const bool isA = wrap ? (j + E < hiA) : (j < hiA);
-    const int idx = (isA ? offA : offB) + (wrap ? j + E : j);
+    const bool isA = (maskA >> j) & 1u;
+    const int idx = (wrap ? (isA ? bAw : bBw) : (isA ? bAn : bBn)) + j;
     bool ok = true;
     if constexpr (!FULL_TILE) {
       const int ia = wrap ? j + E - k : j - k;

@@ -190,10 +190,16 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
       vk[r] = PAD_KEY;
       vv[r] = 0;
       if (p < cnt) {
-        uint32_t x = __ldg(gin_k + p);
-        if (args.encode_f32) x = f32_encode(x);
-        vk[r] = x;
+        vk[r] = __ldg(gin_k + p);
         if constexpr (PAIRS) vv[r] = __ldg(gin_v + p);
+      }
+    }
+    if (args.encode_f32) {
+#pragma unroll
+      for (int r = 0; r < E; ++r) {
+        const int P = tid + r * U;
+        const int p = CF ? rho_inv<E>(P) : P;
+        if (p < cnt) vk[r] = f32_encode(vk[r]);
       }
     }
 #pragma unroll
@@ -226,13 +232,32 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
     if constexpr (CF) {
       // conflict-free scatter (fn. 5): B runs are written
       // reversed (pi); in round m B-run lanes write item E-1-m so that every
-      // lane writes logical index = m (mod E).
+      // lane writes logical index = m (mod E).  From l = 5 on a run spans
+      // whole warps, so the A/B choice is warp-uniform.
       const int base = isB ? gbase + 2 * S - E - ir * E : gbase + ir * E;
+      if ((1 << l) >= W) {
+        if (isB) {
 #pragma unroll
-      for (int m = 0; m < E; ++m) {
-        const int idx = rho<E>(base + m);
-        sk[idx] = isB ? key[E - 1 - m] : key[m];
-        if constexpr (PAIRS) sv[idx] = isB ? val[E - 1 - m] : val[m];
+          for (int m = 0; m < E; ++m) {
+            const int idx = rho<E>(base + m);
+            sk[idx] = key[E - 1 - m];
+            if constexpr (PAIRS) sv[idx] = val[E - 1 - m];
+          }
+        } else {
+#pragma unroll
+          for (int m = 0; m < E; ++m) {
+            const int idx = rho<E>(base + m);
+            sk[idx] = key[m];
+            if constexpr (PAIRS) sv[idx] = val[m];
+          }
+        }
+      } else {
+#pragma unroll
+        for (int m = 0; m < E; ++m) {
+          const int idx = rho<E>(base + m);
+          sk[idx] = isB ? key[E - 1 - m] : key[m];
+          if constexpr (PAIRS) sv[idx] = isB ? val[E - 1 - m] : val[m];
+        }
       }
     } else {
       const int base = gbase + (isB ? S : 0) + ir * E;

@@ -42,3 +42,17 @@ for c in [ctas[0], ctas[len(ctas)//3], ctas[2*len(ctas)//3]]:
             break
         f = lambda v: "%7.2f" % ((v - t0) / 1e3) if v else "      -"
         print(f"  tile {i}: split_known {f(row[128+4*i+1])} empty_ok {f(row[128+4*i+3])} load_issued {f(row[128+4*i+2])} | wait {f(row[1+4*i])} ready {f(row[2+4*i])} done {f(row[3+4*i])}")
+ends = []
+starts = []
+for c in ctas:
+    row = tr[c]
+    done = [row[3 + 4 * i] for i in range(60) if row[3 + 4 * i]]
+    if done:
+        ends.append((max(done) - t0) / 1e3)
+    r0 = [row[2 + 4 * i] for i in range(1)]
+    starts.append((row[2] - t0) / 1e3)
+ends = np.array(ends)
+print("CTA finish us: min %.1f p10 %.1f p50 %.1f p90 %.1f max %.1f" % tuple(np.percentile(ends, [0, 10, 50, 90, 100])))
+print("first data ready us: min %.1f p50 %.1f max %.1f" % tuple(np.percentile(starts, [0, 50, 100])))
+ntile = [sum(1 for i in range(60) if tr[c][3 + 4 * i]) for c in ctas]
+print("tiles per CTA: min %d max %d" % (min(ntile), max(ntile)))
