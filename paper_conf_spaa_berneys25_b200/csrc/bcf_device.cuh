@@ -464,6 +464,20 @@ __device__ __forceinline__ void merge_registers(uint32_t (&key)[E], uint32_t (&v
       }
     }
     bitonic_merge_pad<E, PAIRS>(key, tag, val);
+  } else if constexpr (cpow2ceil(E) == E + 1 && !PAIRS) {
+    // keys only, N = E + 1: append a copy X of register E-1 at slot E.  In the
+    // circular order slot E sits between registers E-1 and 0, and X equals
+    // one of its neighbours, so the 16 slots stay (circularly) bitonic.  After
+    // the merger, drop one copy of X: out[i] = s[i] if s[i] < X else s[i+1].
+    constexpr int N = E + 1;
+    uint32_t K[N], Tg[N], V[N];
+#pragma unroll
+    for (int m = 0; m < E; ++m) K[m] = key[m];
+    K[E] = key[E - 1];
+    const uint32_t X = key[E - 1];
+    bitonic_merge_pad<N, false>(K, Tg, V);
+#pragma unroll
+    for (int i = 0; i < E; ++i) key[i] = K[i] < X ? K[i] : K[i + 1];
   } else if constexpr (cpow2ceil(E) == E + 1) {
     // N = E + 1: insert one minimum element (key 0, tag 0; real tags shift
     // by 1) at register k, i.e. between the circular minimum candidates
