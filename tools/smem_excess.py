@@ -16,7 +16,7 @@ for r in rows:
     if r[0] == "File Path":
         fpath = r[1].split("/")[-1]; continue
     if r[0] == "Function Name":
-        func = r[1].split("(")[0].replace("void bcf::", "")[:60]; continue
+        func = r[1].replace("void bcf::", "").split(">(")[0] + ">"; continue
     if r[0] == "Line No":
         continue
     if r[0]:
