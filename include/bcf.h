@@ -59,8 +59,8 @@ typedef enum {
 } bcf_algo;
 
 /* "software parameters" E and u: items per thread and threads
-   per block.  0 selects the default.  Instantiated set: E in [7, 17],
-   u in {128, 256, 512}. */
+   per block.  0 selects the default.  Instantiated set: E in [7, 17] or
+   E = 31, u in {128, 256, 512}. */
 typedef struct {
   int32_t items_per_thread; /* E */
   int32_t block_threads;    /* u */

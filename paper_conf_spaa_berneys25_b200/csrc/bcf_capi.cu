@@ -38,16 +38,18 @@ LaunchTable& launch_table() {
     register_E15(*p);
     register_E16(*p);
     register_E17(*p);
+    register_E31(*p);
     return p;
   }();
   return *t;
 }
 
-// Defaults for sm_100a: E = 16 makes the in-register
-// merge a pure 16-wide bitonic merger (no rotation) and the tile a power of
-// two; rho (d = 16) keeps every shared-memory access conflict-free.
-static constexpr int DEFAULT_E = 15;
-static constexpr int DEFAULT_U = 256;
+// Defaults for sm_100a (measured by the E/u sweep):
+// E = 31 is coprime with w = 32 (rho = identity, TMA-staged tiles) and
+// E + 1 = 32 makes the in-register merge one 32-wide bitonic merger; u = 128
+// keeps the tile (3968 keys) and the per-thread registers within budget.
+static constexpr int DEFAULT_E = 31;
+static constexpr int DEFAULT_U = 128;
 
 // ---------------------------------------------------------------------------
 // errors, profiler, launch accounting
@@ -108,7 +110,8 @@ static bcf_status resolve(const bcf_params* p, Params& out) {
   out.U = (p && p->block_threads) ? p->block_threads : DEFAULT_U;
   out.algo = p ? p->algo : BCF_ALGO_CONFLICT_FREE;
   if (out.algo != BCF_ALGO_CONFLICT_FREE && out.algo != BCF_ALGO_BASELINE) return BCF_ERROR_INVALID_VALUE;
-  if (out.E < E_MIN || out.E > E_MAX || u_index(out.U) < 0) return BCF_ERROR_UNSUPPORTED;
+  if (out.E < E_MIN || out.E > E_MAX || (out.E > 17 && out.E != 31) || u_index(out.U) < 0)
+    return BCF_ERROR_UNSUPPORTED;
   return BCF_SUCCESS;
 }
 

@@ -20,7 +20,7 @@ struct Variant {
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]
-constexpr int E_MIN = 7, E_MAX = 17;
+constexpr int E_MIN = 7, E_MAX = 31;
 struct LaunchTable {
   Variant v[E_MAX + 1][3][2][2];
 };
@@ -43,6 +43,7 @@ BCF_DECLARE_REG(14)
 BCF_DECLARE_REG(15)
 BCF_DECLARE_REG(16)
 BCF_DECLARE_REG(17)
+BCF_DECLARE_REG(31)
 #undef BCF_DECLARE_REG
 
 }  // namespace bcf

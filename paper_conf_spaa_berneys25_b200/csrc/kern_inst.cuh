@@ -8,23 +8,26 @@
 
 namespace bcf {
 
-// Opt in to > 48 KB dynamic shared memory once per (kernel, device).
+// Opt in to > 48 KB dynamic shared memory once per (kernel, device).  The
+// once-flag must be distinct per kernel instantiation: it lives in the
+// caller's template (not in a helper templated only on the function type).
 template <typename K>
-cudaError_t ensure_smem_attr(K kernel, size_t bytes) {
-  static int done_mask = 0;  // bit per device ordinal (< 32 devices)
+cudaError_t ensure_smem_attr(K kernel, size_t bytes, int& done_mask) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (bytes <= 48 * 1024 || (__atomic_load_n(&done_mask, __ATOMIC_ACQUIRE) >> dev) & 1) return cudaSuccess;
   e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   if (e == cudaSuccess) __atomic_fetch_or(&done_mask, 1 << dev, __ATOMIC_ACQ_REL);
+  else (void)cudaGetLastError();  // do not leave a stale error for the next launch check
   return e;
 }
 
 template <int E, int U, bool PAIRS, bool CF>
 cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
-  cudaError_t e = ensure_smem_attr(block_sort_kernel<E, U, PAIRS, CF>, smem);
+  static int done = 0;
+  cudaError_t e = ensure_smem_attr(block_sort_kernel<E, U, PAIRS, CF>, smem, done);
   if (e != cudaSuccess) return e;
   block_sort_kernel<E, U, PAIRS, CF><<<(unsigned)grid, U, smem, s>>>(a);
   return cudaGetLastError();
@@ -33,7 +36,8 @@ cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s)
 template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
-  cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, smem);
+  static int done = 0;
+  cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, smem, done);
   if (e != cudaSuccess) return e;
   merge_pass_kernel<E, U, PAIRS, CF, BDESC><<<(unsigned)grid, U, smem, s>>>(a);
   return cudaGetLastError();
@@ -56,7 +60,10 @@ cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int thre
   if (pc.per_sm[dev] == 0) {
     if (smem > 48 * 1024) {
       e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      if (e != cudaSuccess) return e;
+      if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        return e;
+      }
     }
     int k = 0, sms = 0;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, threads, smem);
@@ -80,7 +87,10 @@ cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int thre
 template <int E, int U, bool PAIRS>
 cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s) {
   static PersistentCache pc;  // one per (E, U, PAIRS) instantiation
-  if constexpr (!PAIRS && BCF_MERGE_WIN) {
+  // the 2-stage window ring needs 2 x 2T words: beyond 227 KB (E = 31,
+  // u = 512) fall back to the 3-stage exact-split TMA kernel
+  constexpr bool win_fits = win_smem_bytes<E, U>() <= 227 * 1024;
+  if constexpr (!PAIRS && BCF_MERGE_WIN && win_fits) {
     return launch_persistent(merge_pass_win_kernel<E, U>, pc, win_smem_bytes<E, U>(), U + 32, a, tiles, s);
   } else {
     return launch_persistent(merge_pass_tma_kernel<E, U, PAIRS>, pc, tma_smem_bytes<E, U, PAIRS>(), U + 32,

@@ -45,8 +45,11 @@ def test_abi_version_and_status_strings():
 
 
 def test_default_params():
+    import bench
+
     p = bcf.default_params()
-    assert 7 <= p.items_per_thread <= 17
+    assert (p.items_per_thread, p.block_threads) == (bench.DEFAULT_E, bench.DEFAULT_U)
+    assert 7 <= p.items_per_thread <= 17 or p.items_per_thread == 31
     assert p.block_threads in (128, 256, 512)
     assert p.algo == bcf.ALGO_CONFLICT_FREE
 
@@ -71,6 +74,9 @@ def test_temp_query_and_validation():
     # unsupported parameters are rejected before any launch
     assert _query(L.bcf_sort_u32, 100, bcf.make_params(6, 256))[0] == bcf.BCF_ERROR_UNSUPPORTED
     assert _query(L.bcf_sort_u32, 100, bcf.make_params(18, 256))[0] == bcf.BCF_ERROR_UNSUPPORTED
+    assert _query(L.bcf_sort_u32, 100, bcf.make_params(30, 256))[0] == bcf.BCF_ERROR_UNSUPPORTED
+    assert _query(L.bcf_sort_u32, 100, bcf.make_params(32, 256))[0] == bcf.BCF_ERROR_UNSUPPORTED
+    assert _query(L.bcf_sort_u32, 100, bcf.make_params(31, 128))[0] == 0
     assert _query(L.bcf_sort_u32, 100, bcf.make_params(15, 384))[0] == bcf.BCF_ERROR_UNSUPPORTED
     assert _query(L.bcf_sort_u32, 100, bcf.make_params(15, 256, 7))[0] == bcf.BCF_ERROR_INVALID_VALUE
     assert _query(L.bcf_sort_pairs_u32, 100, bcf.make_params(15, 256, bcf.ALGO_BASELINE),
@@ -99,6 +105,7 @@ def test_temp_query_and_validation():
     (15, 64, 15 * 2 ** 9, 1234), (17, 64, 17 * 2 ** 9, 5), (16, 64, 2 ** 13, 7), (12, 64, 12 * 2 ** 9, 9),
     (8, 128, 2 ** 13, 11), (15, 256, 100000, 3), (16, 256, 2 ** 16, 0xB2000000), (9, 128, 7777, 1),
     (13, 512, 1, 2), (7, 128, 0, 3), (15, 512, 15 * 2 ** 14, 4), (11, 256, 50001, 8),
+    (31, 128, 31 * 2 ** 12, 6), (31, 128, 100001, 7),
 ])
 def test_host_worst_case_matches_oracle(E, u, n, seed):
     got = bcf.worst_case_host(n, E, u, seed)

@@ -46,7 +46,7 @@ def test_default_u32_parity(n, kind):
     np.testing.assert_array_equal(gpu_sort_u32(x), oracle.sort_u32(x))
 
 
-@pytest.mark.parametrize("E", list(range(7, 18)))
+@pytest.mark.parametrize("E", list(range(7, 18)) + [31])
 @pytest.mark.parametrize("u", [128, 256, 512])
 @pytest.mark.parametrize("algo", [bcf.ALGO_CONFLICT_FREE, bcf.ALGO_BASELINE])
 def test_all_instantiations_u32(E, u, algo):
@@ -103,7 +103,7 @@ def test_f32_uniform():
     np.testing.assert_array_equal(got, oracle.sort_f32_bits(x.view(np.uint32)))
 
 
-@pytest.mark.parametrize("E,u", [(16, 256), (15, 256), (17, 128), (8, 512), (12, 256), (7, 128), (16, 512)])
+@pytest.mark.parametrize("E,u", [(16, 256), (15, 256), (17, 128), (8, 512), (12, 256), (7, 128), (16, 512), (31, 128)])
 @pytest.mark.parametrize("n", [1, 17, 4097, 100000])
 def test_pairs_stable(E, u, n):
     k = si.dup_u32(n, si.config_seed(4) + n, mask=0xF)
