@@ -17,6 +17,7 @@
 // ascending.  The baseline keeps every run ascending.
 #pragma once
 #include "bcf_device.cuh"
+#include "bcf_tma.cuh"
 
 namespace bcf {
 
@@ -176,6 +177,7 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   const long long t0 = tile * T;
   const long long rem = args.n - t0;
   const int cnt = rem < T ? (int)rem : T;
+  tma::pdl_wait();  // the input may be produced by the preceding grid
 
   // --- load: coalesced in physical order, pads = max key (they sort last and
   // are trimmed by the count; stable order keeps them after real max keys).
@@ -312,6 +314,7 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
     }
   }
   __syncthreads();
+  tma::pdl_trigger();  // the next pass may be scheduled once this wave ends
   // --- store run `tile`: descending iff tile odd (CF directions)
   const bool desc = args.cf_dirs && (tile & 1);
   // a short descending run is stored shifted by sigma = (T - cnt) mod 4
@@ -337,6 +340,7 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   const int lane = tid & (W - 1);
   const int warp = tid >> 5;
   const long long tile = blockIdx.x;
+  tma::pdl_wait();  // pass i reads what pass i-1 wrote (and overwrites what it read)
   long long j;
   const GroupDesc grp = group_of_tile(args, tile, T, j);
   const long long lenG = grp.na + grp.nb;
@@ -454,6 +458,7 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
     }
   }
   __syncthreads();
+  tma::pdl_trigger();
   // --- output tile into the group's output run (descending if grp.out_desc)
   const bool desc = grp.out_desc != 0;
   const long long c0 = desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;

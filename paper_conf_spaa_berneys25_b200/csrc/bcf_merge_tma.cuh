@@ -68,6 +68,22 @@ __device__ __forceinline__ unsigned long long gtimer() {
     if (args.trace && (slot) < 256) args.trace[(size_t)blockIdx.x * 256 + (slot)] = gtimer(); \
   } while (0)
 
+// tiles [t_begin, t_end) of this CTA: per_cta > 0 -> fixed chunks of per_cta
+// tiles; per_cta == 0 -> the tiles spread evenly over the grid (chunks differ
+// by at most one tile, so a grid of SMs x resident CTAs is load-balanced)
+__device__ __forceinline__ void cta_tile_range(long long tiles, long long per_cta, long long& t_begin,
+                                               long long& t_end) {
+  const long long b = blockIdx.x;
+  if (per_cta > 0) {
+    t_begin = b * per_cta;
+    t_end = t_begin + per_cta;
+  } else {
+    t_begin = b * tiles / gridDim.x;
+    t_end = (b + 1) * tiles / gridDim.x;
+  }
+  if (t_end > tiles) t_end = tiles;
+}
+
 __device__ __forceinline__ int align_up4(int x) { return (x + 3) & ~3; }
 __device__ __forceinline__ int align_dn4(int x) { return x & ~3; }
 
@@ -151,9 +167,8 @@ __global__ void __launch_bounds__(U + 32, BCF_TMA_MINB) merge_pass_tma_kernel(Me
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   const int lane = tid & (W - 1);
-  const long long t_begin = (long long)blockIdx.x * per_cta;
-  long long t_end = t_begin + per_cta;
-  if (t_end > tiles) t_end = tiles;
+  long long t_begin, t_end;
+  cta_tile_range(tiles, per_cta, t_begin, t_end);
   const int m = (int)(t_end - t_begin);
   if (m <= 0) return;  // uniform over the CTA
 
@@ -166,6 +181,8 @@ __global__ void __launch_bounds__(U + 32, BCF_TMA_MINB) merge_pass_tma_kernel(Me
       tma::mbar_init(&empty_bar[s], 1);
     }
   }
+  tma::pdl_wait();     // pass i reads what pass i-1 wrote (and overwrites what it read)
+  tma::pdl_trigger();  // one persistent wave: the next pass may queue for our slots
   // Startup: the NW + 1 warps compute, in parallel, the merge-path
   // boundaries of the first tiles of the chunk (full-range 64-ary searches):
   // s_bnd[k] = a(start of tile k) for k < min(m, NW + 1), and

@@ -1,28 +1,41 @@
-// bcf_merge_win.cuh -- persistent CF merge pass with self-splitting tiles
-// (keys only, E coprime with 32).
+// bcf_merge_win.cuh -- persistent CF merge pass with self-splitting,
+// variable-size tiles (keys only, E coprime with 32).
 //
-// A CTA (NW consumer warps + 1 producer warp) walks a contiguous chunk of
-// output tiles.  Tile i starts at the merge-path point (a0, b0) -- known from
-// the previous tile -- and the producer bulk-loads (TMA) a WINDOW of T keys
-// of A from a0 and T keys of B from b0 into a 2-stage shared ring, laid out
-// as the paper's rho(A u pi(B)) over a span of 2T (A at [0, WA), B reversed
-// at [2T - WB, 2T); 2T is a multiple of wE, so every round set of §3.3 is
-// unchanged).  The first T outputs only involve keys inside the windows, so
-// the consumers find the tile's own end split a(T) in shared memory (warp 0,
-// conflict-free 32-ary search) while the other warps compute their origins;
-// warp 0 publishes the split through an mbarrier and the producer
-// immediately bulk-loads the next tile's window.  The window data beyond the
-// tile is re-read by the next tile from L2 (DRAM traffic stays ~8 B/key).
-// The only global merge-path search left is the first boundary of a chunk
-// that starts inside a merge group.
+// A CTA (NW consumer warps + 1 producer warp) walks a contiguous range of the
+// pass's output (the tiles [t_begin, t_end) of T = U*E outputs each) as a
+// sequence of SUBTILES of at most T outputs.  Subtile i starts at the
+// merge-path point (a0, b0) -- known from subtile i-1 -- and the producer
+// bulk-loads (TMA) a window of WA keys of A from a0 and WB keys of B from b0
+// into a 2-stage shared ring.  The stage is the paper's rho(A u pi(B)) over a
+// span of S2 = T + T/4 words (A at [0, WA), B reversed at [S2 - WB, S2); S2
+// is a multiple of wE, so every round set of §3.3 is unchanged), with
+// WA + WB = S2: the split of the span between A and B is predicted from the
+// previous subtile's A share.  The first outputs of the merge only involve
+// keys inside the windows, so the consumers find the subtile's own end split
+// in shared memory (warp 0, conflict-free k-ary search), and if the merge path
+// leaves a window before T outputs (a badly predicted or skewed split) the
+// subtile simply ends there, at a multiple of 4 outputs (the rare path).  Warp 0
+// publishes (count, split) through an mbarrier and the producer immediately
+// bulk-loads the next window.  A span of 1.25 T instead of 2 T (one window
+// of T keys per run) keeps five CTAs resident per SM for (E, u) = (31, 128).
+// The only global merge-path search left is the first boundary of a CTA's
+// range when it starts inside a merge group.
 #pragma once
 #include "bcf_merge_tma.cuh"
 
 namespace bcf {
 
+#ifndef BCF_WIN_Q
+#define BCF_WIN_Q 1  // span S2 = T + Q * T/4 (Q = 4: two full windows, never exhausted)
+#endif
+
+template <int E, int U>
+__host__ __device__ constexpr int win_span() {
+  return U * E + BCF_WIN_Q * (U / 4) * E;  // U/4 is a multiple of w: S2 = 0 (mod wE)
+}
 template <int E, int U>
 __host__ __device__ constexpr int win_stage_words() {
-  return ((2 * U * E + E + 8) + 3) / 4 * 4;  // 2T + cell-scan slack + shift
+  return ((win_span<E, U>() + E + 8) + 3) / 4 * 4;  // span + cell-scan slack + shift
 }
 constexpr int WIN_STAGES = 2;
 template <int E, int U>
@@ -33,34 +46,57 @@ __host__ __device__ constexpr size_t win_smem_bytes() {
 struct WinMeta {
   long long c0;       // output global word of logical output index q
   int WA, WB;         // window sizes (keys of A / B present)
-  int cnt, c, cout, qlo, qhi, desc;
-  int NA;             // tile's A count, written by the consumers
+  int cmax;           // outputs wanted (<= T); the consumers may end earlier
+  int fin;            // bit 0: A window holds every A key the subtile can need; bit 1: B
+  int c, cout, desc, exit;
+  int NA, cnt;        // the subtile's A count and output count (consumers)
 };
+
+// Number of leading elements of a sorted window for which pred holds
+// (pred true on a prefix).  Warp-cooperative 32-ary search; the probes of one
+// round are at an odd stride, i.e. distinct banks for consecutive storage (or
+// reversed consecutive storage) under rho = identity.
+template <class P>
+__device__ __forceinline__ int warp_prefix_count(int n, P pred, int lane) {
+  int lo = 0, hi = n;
+  while (hi > lo) {
+    const int s = (((hi - lo) + 31) >> 5) | 1;
+    const int m = lo + (lane + 1) * s - 1;
+    const bool p = m < hi && pred(m);
+    const int c = __popc(__ballot_sync(FULL, p));
+    const int nlo = lo + c * s;
+    int nhi = lo + (c + 1) * s - 1;
+    if (nhi > hi) nhi = hi;
+    lo = nlo;
+    hi = nhi;
+    if (s == 1) break;
+  }
+  return lo;
+}
 
 template <int E, int U>
 __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, long long tiles,
                                                                 long long per_cta) {
   constexpr int T = U * E;
-  constexpr int T2 = 2 * T;
+  constexpr int S2 = win_span<E, U>();
   constexpr int NW = U / W;
   constexpr int SW = win_stage_words<E, U>();
   constexpr int S = WIN_STAGES;
   static_assert(cgcd(W, E) == 1, "window staging needs rho = identity (E coprime with 32)");
+  static_assert(S2 % (W * E) == 0 && S2 % 4 == 0 && S2 > T, "span must be a multiple of wE");
   extern __shared__ __align__(16) uint32_t smem_dyn[];
   __shared__ WinMeta meta[S];
   __shared__ __align__(8) uint64_t full_bar[S];
   __shared__ __align__(8) uint64_t empty_bar[S];
   __shared__ __align__(8) uint64_t split_bar[S];
-  __shared__ int s_org[NW + 1];
+  __shared__ int s_org[NW + 2];
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   const int lane = tid & (W - 1);
-  const long long t_begin = (long long)blockIdx.x * per_cta;
-  long long t_end = t_begin + per_cta;
-  if (t_end > tiles) t_end = tiles;
-  const int m = (int)(t_end - t_begin);
-  if (m <= 0) return;
+  long long t_begin, t_end;
+  cta_tile_range(tiles, per_cta, t_begin, t_end);
+  if (t_end <= t_begin) return;
   auto stage = [&](int s) { return smem_dyn + (size_t)s * SW; };
 
   if (tid == 0) {
@@ -71,45 +107,82 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
     }
   }
   __syncthreads();
+  tma::pdl_wait();     // pass i reads what pass i-1 wrote (and overwrites what it read)
+  tma::pdl_trigger();  // one persistent wave: the next pass may queue for our slots
 
   if (warp == NW) {
     // =========================== producer ===========================
     const uint32_t* __restrict__ src = args.src_k;
     const long long dst_phase = (long long)(((uintptr_t)args.dst_k >> 2) & 3);
 
-    // window load of tile t starting at merge-path point a0 into stage s
-    auto load_window = [&](int s, long long t, long long a0) {
-      long long j;
-      const GroupDesc grp = group_of_tile(args, t, T, j);
+    // current segment: the part of one merge group inside this CTA's range
+    long long j0;
+    GroupDesc grp = group_of_tile(args, t_begin, T, j0);
+    auto seg_end = [&](const GroupDesc& g, long long tile0) {
+      const long long lenG = g.na + g.nb;
+      long long te = g.tile_begin + (lenG + T - 1) / T;
+      if (te > t_end) te = t_end;
+      long long De = (te - g.tile_begin) * T;
+      return De < lenG ? De : lenG;
+    };
+    long long Dend = seg_end(grp, t_begin);
+    long long D0 = j0 * T;
+    long long a0;
+    {
+      RunView Av{src + grp.a_off, grp.na, 0};
+      RunView Bv{src + grp.b_off, grp.nb, 1};
       const long long lenG = grp.na + grp.nb;
-      const long long D0 = j * T;
+      const long long guess = lenG > 0 ? (long long)((double)D0 * (double)grp.na / (double)lenG) : 0;
+      a0 = j0 == 0 ? 0 : merge_path_warp_global_guess(Av, Bv, D0, 0, D0, guess, lane);
+    }
+    // predicted A share of the next subtile (fraction of outputs, x 2^16)
+    int shareA = (grp.na + grp.nb) > 0 ? (int)((grp.na << 16) / (grp.na + grp.nb)) : 32768;
+
+    // subtile window of the current (grp, D0, a0) into stage s
+    auto load_window = [&](int s) {
+      const long long lenG = grp.na + grp.nb;
       const long long b0 = D0 - a0;
       WinMeta M;
-      const long long cnt = lenG - D0 < T ? lenG - D0 : T;
-      M.cnt = (int)cnt;
-      M.WA = (int)(grp.na - a0 < T ? grp.na - a0 : T);
-      M.WB = (int)(grp.nb - b0 < T ? grp.nb - b0 : T);
+      const int cmax = (int)(Dend - D0 < T ? Dend - D0 : T);
+      const long long remA = grp.na - a0, remB = grp.nb - b0;
+      const int needA = (int)(remA < cmax ? remA : cmax);
+      const int needB = (int)(remB < cmax ? remB : cmax);
+      int WA, WB;
+      if (needA + needB <= S2) {
+        WA = needA;
+        WB = needB;
+      } else {
+        // predicted A count + half the slack, clamped so that both windows fit
+        int pa = (int)(((long long)shareA * cmax) >> 16) + (S2 - cmax) / 2;
+        const int lo = S2 - needB, hi = needA;
+        pa = pa < lo ? lo : (pa > hi ? hi : pa);
+        WA = pa;
+        WB = S2 - pa;
+      }
+      M.WA = WA;
+      M.WB = WB;
+      M.cmax = cmax;
+      M.fin = (WA == needA ? 1 : 0) | (WB == needB ? 2 : 0);
+      M.exit = 0;
       const long long oA = grp.a_off + a0;                  // A[a0 + q] at word oA + q
-      const long long oB = grp.b_off + grp.nb - b0 - T2;    // logical q (B part) at oB + q
+      const long long oB = grp.b_off + grp.nb - b0 - S2;    // logical q (B part) at oB + q
       const int c = (int)(oA & 3);
       M.c = c;
       M.desc = grp.out_desc;
       M.c0 = M.desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
-      M.qlo = M.desc ? T - M.cnt : 0;
-      M.qhi = M.desc ? T : M.cnt;
       M.cout = (int)((unsigned long long)(dst_phase + M.c0) & 3ull);
       M.NA = 0;
+      M.cnt = 0;
       if (lane == 0) meta[s] = M;
-      const int WA = M.WA, WB = M.WB;
       int a_hi = WA ? align_up4(c + WA) : 0;
-      int b_lo = WB ? align_dn4(c + T2 - WB) : 0;
-      const int b_hi = WB ? align_up4(c + T2) : 0;
+      int b_lo = WB ? align_dn4(c + S2 - WB) : 0;
+      const int b_hi = WB ? align_up4(c + S2) : 0;
       int ea0 = 0, ea1 = 0, eb0 = 0, eb1 = 0;
       if (WA && WB && a_hi > b_lo) {
         ea1 = c + WA;
         a_hi = align_dn4(ea1);
         ea0 = a_hi;
-        eb0 = c + T2 - WB;
+        eb0 = c + S2 - WB;
         b_lo = align_up4(eb0);
         eb1 = b_lo;
       }
@@ -124,52 +197,81 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
         w = eb0 + lane - 4;
         gw = oB + (w - c);
       }
-      const uint32_t ev = w >= 0 ? __ldg(src + gw) : 0u;
       if (lane == 0) {
         tma::mbar_expect_tx(&full_bar[s], (uint32_t)(a_hi + (b_hi - b_lo)) * 4u);
         if (a_hi > 0) tma::bulk_g2s(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
         if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, src + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        // L2 prefetch of the keys the next window will need beyond this one
+        // (both runs are consumed sequentially): the next window's bulk loads,
+        // issued one subtile later, then hit L2 instead of DRAM
+        constexpr long long PF = (3 * T / 4 + 3) & ~3;
+        const long long pa0 = (oA + WA + 3) & ~3ll;                  // A: ascending words
+        long long pa1 = grp.a_off + grp.na;
+        if (pa1 > pa0 + PF) pa1 = pa0 + PF;
+        pa1 &= ~3ll;
+        if (pa1 > pa0) tma::bulk_prefetch_l2(src + pa0, (uint32_t)(pa1 - pa0) * 4u);
+        long long pb1 = (grp.b_off + grp.nb - b0 - WB) & ~3ll;      // B: descending words
+        long long pb0 = grp.b_off;
+        if (pb0 < pb1 - PF) pb0 = pb1 - PF;
+        pb0 = (pb0 + 3) & ~3ll;
+        if (pb1 > pb0) tma::bulk_prefetch_l2(src + pb0, (uint32_t)(pb1 - pb0) * 4u);
       }
+      const uint32_t ev = w >= 0 ? __ldg(src + gw) : 0u;
       if (w >= 0) sk[w] = ev;
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);
-      return grp.tile_begin;
+    };
+    auto post_exit = [&](int s) {
+      if (lane == 0) {
+        meta[s].exit = 1;
+        tma::mbar_arrive(&full_bar[s]);
+      }
+      __syncwarp();
     };
 
-    // chunk start: the only global merge-path search
-    long long a0;
-    {
-      long long j;
-      const GroupDesc grp = group_of_tile(args, t_begin, T, j);
-      const long long D0 = j * T;
-      RunView Av{src + grp.a_off, grp.na, 0};
-      RunView Bv{src + grp.b_off, grp.nb, 1};
-      a0 = j == 0 ? 0 : merge_path_warp_global_bounded(Av, Bv, D0, 0, D0, lane);
-    }
     if (lane == 0) BCF_TRACE_AT(0);
-    long long tb = load_window(0, t_begin, a0);
+    if (lane == 0 && args.trace) {
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      args.trace[(size_t)blockIdx.x * 256 + 255] = smid + 1;
+    }
+    load_window(0);
     if (lane == 0) BCF_TRACE_AT(128 + 2);
-    for (int i = 0; i < m; ++i) {
+    for (int i = 0;; ++i) {
       const int s = i % S;
-      const uint32_t u = (uint32_t)(i / S);
-      // tile i's own end split, found by its consumers
-      tma::mbar_wait(&split_bar[s], u & 1);
-      if (lane == 0) BCF_TRACE_AT(128 + 4 * i + 1);
-      const int NA = meta[s].NA;
-      if (i + 1 < m) {
-        long long j1;
-        const GroupDesc g1 = group_of_tile(args, t_begin + i + 1, T, j1);
-        const long long a_next = (g1.tile_begin == tb) ? a0 + NA : 0;
-        const int s1 = (i + 1) % S;
-        if (i >= 1) {
-          // stage s1 held tile i-1: its consumers must have copied it out
-          tma::mbar_wait(&empty_bar[s1], (uint32_t)((i - 1) / S) & 1);
-          if (lane == 0) BCF_TRACE_AT(128 + 4 * (i + 1) + 3);
+      // subtile i's own end split, found by its consumers
+      tma::mbar_wait(&split_bar[s], (uint32_t)(i / S) & 1);
+      if (lane == 0 && i < 7) BCF_TRACE_AT(128 + 4 * i + 1);
+      const int NA = meta[s].NA, cnt = meta[s].cnt;
+      if (cnt > 0) shareA = (int)(((long long)NA << 16) / cnt);
+      D0 += cnt;
+      a0 += NA;
+      bool more = true;
+      if (D0 >= Dend) {
+        // segment done: the next one starts a new merge group at its first tile
+        const long long tn = grp.tile_begin + (Dend + T - 1) / T;
+        if (tn >= t_end) {
+          more = false;
+        } else {
+          grp = group_of_tile(args, tn, T, j0);
+          Dend = seg_end(grp, tn);
+          D0 = 0;
+          a0 = 0;
+          shareA = (grp.na + grp.nb) > 0 ? (int)((grp.na << 16) / (grp.na + grp.nb)) : 32768;
         }
-        a0 = a_next;
-        tb = load_window(s1, t_begin + i + 1, a0);
-        if (lane == 0) BCF_TRACE_AT(128 + 4 * (i + 1) + 2);
       }
+      const int s1 = (i + 1) % S;
+      if (i >= 1) {
+        // stage s1 held subtile i-1: its consumers must have copied it out
+        tma::mbar_wait(&empty_bar[s1], (uint32_t)((i - 1) / S) & 1);
+        if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 3);
+      }
+      if (!more) {
+        post_exit(s1);
+        break;
+      }
+      load_window(s1);
+      if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 2);
     }
     return;
   }
@@ -177,32 +279,57 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
   // ============================ consumers ============================
   const bool decode = args.decode_f32 != 0;
   uint32_t dummy[E];
-  for (int i = 0; i < m; ++i) {
+  for (int i = 0;; ++i) {
     const int s = i % S;
-    if (tid == 0) BCF_TRACE_AT(1 + 4 * i);
+    if (tid == 0 && i < 31) BCF_TRACE_AT(1 + 4 * i);
     tma::mbar_wait(&full_bar[s], (uint32_t)(i / S) & 1);
-    if (tid == 0) BCF_TRACE_AT(2 + 4 * i);
+    if (tid == 0 && i < 31) BCF_TRACE_AT(2 + 4 * i);
     const WinMeta M = meta[s];
+    if (M.exit) break;
     uint32_t* sk = stage(s) + M.c;  // logical index -> sk[index]
-    const int WA = M.WA, WB = M.WB, cnt = M.cnt;
+    const int WA = M.WA, WB = M.WB, cmax = M.cmax;
     const int D = tid * E;
     const int Dw = warp * W * E;
-    // warp 0: the tile's end split a(cnt) (its own origin is 0); other warps:
-    // their origins a(Dw).  Window bounds are exact for every D <= cnt.
-    const int probe = warp == 0 ? cnt : Dw;
-    const int r = warp_origin_smem<E>(sk, 0, T2, WA, WB, probe, lane);
+    // warp 0: the subtile's end split a(cmax) (its own origin is 0); other
+    // warps: their origins a(Dw).  The window path equals the merge path as
+    // long as neither window is exhausted early.
+    const int probe = warp == 0 ? cmax : Dw;
+    int r = warp_origin_smem<E>(sk, 0, S2, WA, WB, probe, lane);
     const int alpha = warp == 0 ? 0 : r;
     if (lane == 0) s_org[warp] = alpha;
-    if (warp == 0 && lane == 0) {
-      s_org[NW] = r;
-      meta[s].NA = r;
-      tma::mbar_arrive(&split_bar[s]);  // release: the producer loads the next window
+    if (warp == 0) {
+      int cnt = cmax;
+      if (!(M.fin & 1) && r == WA) {
+        // A window exhausted at D_A = WA + #{B[y] < A[WA-1]} (ties go to A)
+        const uint32_t v = sk[WA - 1];
+        const int nb = warp_prefix_count(WB, [&](int y) { return sk[S2 - 1 - y] < v; }, lane);
+        cnt = WA + nb;
+      } else if (!(M.fin & 2) && cmax - r == WB) {
+        // B window exhausted at D_B = WB + #{A[x] <= B[WB-1]}
+        const uint32_t v = sk[S2 - WB];
+        const int na = warp_prefix_count(WA, [&](int x) { return !(v < sk[x]); }, lane);
+        cnt = WB + na;
+      }
+      if (cnt < cmax) {
+        // end on a multiple of 4 outputs (16-byte phase of the next windows)
+        cnt &= ~3;
+        r = warp_origin_smem<E>(sk, 0, S2, WA, WB, cnt, lane);
+      }
+      if (lane == 0) {
+        s_org[NW] = r;
+        s_org[NW + 1] = cnt;
+        meta[s].NA = r;
+        meta[s].cnt = cnt;
+        tma::mbar_arrive(&split_bar[s]);  // release: the producer loads the next window
+      }
     }
     tma::named_bar_sync(1, U);
-    // splits past the tile's last output are a(cnt) = NA (windows extend
-    // beyond the tile, so they must be clamped explicitly)
+    if (tid == 0 && i < 30) BCF_TRACE_AT(161 + 3 * i);
+    // splits past the subtile's last output are a(cnt) = NA (windows extend
+    // beyond it, so they must be clamped explicitly)
     const int NA = s_org[NW];
-    int a = lane_split_smem<E>(sk, 0, T2, WA, WB, Dw, alpha, lane, W, 5);
+    const int cnt = s_org[NW + 1];
+    int a = lane_split_smem<E>(sk, 0, S2, WA, WB, Dw, alpha, lane, W, 5);
     if (D >= cnt) a = NA;
     int anext = __shfl_down_sync(FULL, a, 1);
     if (lane == W - 1) anext = (warp + 1) * W * E >= cnt ? NA : s_org[warp + 1];
@@ -213,15 +340,16 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
     const int b = Dc - a;
     uint32_t key[E];
     if (cnt == T)
-      dual_subsequence_gather<E, false, true>(sk, sk, 0, T2, a, b, nA, nB, key, dummy, PAD_KEY);
+      dual_subsequence_gather<E, false, true>(sk, sk, 0, S2, a, b, nA, nB, key, dummy, PAD_KEY);
     else
-      dual_subsequence_gather<E, false, false>(sk, sk, 0, T2, a, b, nA, nB, key, dummy, PAD_KEY);
+      dual_subsequence_gather<E, false, false>(sk, sk, 0, S2, a, b, nA, nB, key, dummy, PAD_KEY);
     merge_registers<E, false>(key, dummy, a, nA, nB);
     if (decode) {
 #pragma unroll
       for (int q = 0; q < E; ++q) key[q] = f32_decode(key[q]);
     }
     tma::named_bar_sync(1, U);  // every consumer has finished reading the stage
+    if (tid == 0 && i < 30) BCF_TRACE_AT(160 + 3 * i);
     uint32_t* ok = stage(s) + M.cout;
     if (M.desc) {
 #pragma unroll
@@ -231,19 +359,22 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
       for (int q = 0; q < E; ++q) ok[D + q] = key[q];
     }
     tma::named_bar_sync(1, U);
-    // copy-out: the tile's outputs sit at stage words [w0, w1), stage word w
-    // belongs at global word g0 + w and both are 16-byte aligned for w = 0
+    if (tid == 0 && i < 31) BCF_TRACE_AT(4 + 4 * i);
+    // copy-out: the subtile's outputs sit at stage words [w0, w1), stage word
+    // w belongs at global word g0 + w and both are 16-byte aligned for w = 0
     // (mod 4): vectorised conflict-free LDS.128 / coalesced STG.128, plus at
     // most 3 + 3 edge words.
     {
-      const int w0 = M.cout + M.qlo, w1 = M.cout + M.qhi;
+      const int qlo = M.desc ? T - cnt : 0;
+      const int qhi = M.desc ? T : cnt;
+      const int w0 = M.cout + qlo, w1 = M.cout + qhi;
       int ilo = align_up4(w0), ihi = align_dn4(w1);
       if (ihi < ilo) ilo = ihi = w1;
       const uint32_t* sb = stage(s);
       uint32_t* gb = args.dst_k + (M.c0 - M.cout);
 #pragma unroll
-      for (int r = 0; r < (T + 4 * U - 1) / (4 * U) + 1; ++r) {
-        const int v = ilo + 4 * (tid + r * U);
+      for (int r2 = 0; r2 < (T + 4 * U - 1) / (4 * U) + 1; ++r2) {
+        const int v = ilo + 4 * (tid + r2 * U);
         if (v < ihi) *reinterpret_cast<uint4*>(gb + v) = *reinterpret_cast<const uint4*>(sb + v);
       }
       const int nh = ilo - w0;
@@ -252,7 +383,7 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
     }
     tma::named_bar_sync(1, U);  // stage reads done: hand it back to the producer
     if (tid == 0) tma::mbar_arrive(&empty_bar[s]);
-    if (tid == 0) BCF_TRACE_AT(3 + 4 * i);
+    if (tid == 0 && i < 31) BCF_TRACE_AT(3 + 4 * i);
   }
 }
 

@@ -88,5 +88,12 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
+// programmatic dependent launch (PDL): wait until the preceding grid in the
+// stream has completed and its memory is visible (no-op without PDL), and
+// allow the next grid to be scheduled once every CTA of this one has called
+// trigger (or exited)
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 }  // namespace tma
 }  // namespace bcf

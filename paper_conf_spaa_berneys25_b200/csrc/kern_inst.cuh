@@ -1,6 +1,8 @@
 // kern_inst.cuh -- explicit instantiation of the kernels for one E and the
 // three block sizes; included by kern_E<E>.cu with BCF_E defined.
 #pragma once
+#include <cstdlib>
+
 #include "bcf_kernels.cuh"
 #include "bcf_merge_tma.cuh"
 #include "bcf_merge_win.cuh"
@@ -23,14 +25,41 @@ cudaError_t ensure_smem_attr(K kernel, size_t bytes, int& done_mask) {
   return e;
 }
 
+// Launch with programmatic dependent launch (PDL): consecutive passes of a
+// sort overlap their launch latency and CTA ramp-up with the previous pass's
+// tail; every kernel waits (griddepcontrol.wait) before touching global
+// memory.  BCF_NO_PDL=1 launches plainly (A/B measurements).
+inline bool pdl_enabled() {
+  static const bool on = [] {
+    const char* v = getenv("BCF_NO_PDL");
+    return !(v && v[0] == '1');
+  }();
+  return on;
+}
+
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*kern)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t s,
+                     Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, args...);
+}
+
 template <int E, int U, bool PAIRS, bool CF>
 cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
   static int done = 0;
   cudaError_t e = ensure_smem_attr(block_sort_kernel<E, U, PAIRS, CF>, smem, done);
   if (e != cudaSuccess) return e;
-  block_sort_kernel<E, U, PAIRS, CF><<<(unsigned)grid, U, smem, s>>>(a);
-  return cudaGetLastError();
+  return launch_k(block_sort_kernel<E, U, PAIRS, CF>, (unsigned)grid, U, smem, s, a);
 }
 
 template <int E, int U, bool PAIRS, bool CF, bool BDESC>
@@ -39,12 +68,11 @@ cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   static int done = 0;
   cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, smem, done);
   if (e != cudaSuccess) return e;
-  merge_pass_kernel<E, U, PAIRS, CF, BDESC><<<(unsigned)grid, U, smem, s>>>(a);
-  return cudaGetLastError();
+  return launch_k(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, (unsigned)grid, U, smem, s, a);
 }
 
 // persistent TMA merge pass: grid = min(tiles, SMs x resident CTAs), each
-// CTA a contiguous chunk of tiles
+// CTA a contiguous, balanced chunk of tiles
 struct PersistentCache {
   int per_sm[32] = {0};
   int nsm[32] = {0};
@@ -73,12 +101,10 @@ cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int thre
     pc.nsm[dev] = sms;
     pc.per_sm[dev] = k > 0 ? k : 1;
   }
+  // one wave of SMs x resident CTAs, tiles spread evenly (per_cta = 0)
   long long ctas = (long long)pc.nsm[dev] * pc.per_sm[dev];
   if (ctas > tiles) ctas = tiles;
-  const long long per_cta = (tiles + ctas - 1) / ctas;
-  ctas = (tiles + per_cta - 1) / per_cta;
-  kern<<<(unsigned)ctas, threads, smem, s>>>(a, tiles, per_cta);
-  return cudaGetLastError();
+  return launch_k(kern, (unsigned)ctas, (unsigned)threads, smem, s, a, tiles, 0ll);
 }
 
 #ifndef BCF_MERGE_WIN

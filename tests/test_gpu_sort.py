@@ -76,6 +76,46 @@ def test_structured_inputs(kind):
     np.testing.assert_array_equal(gpu_sort_u32(x), oracle.sort_u32(x))
 
 
+def _skewed(kind: str, n: int, seed: int) -> np.ndarray:
+    """Inputs whose merge paths leave the predicted windows of the persistent
+    merge pass (bcf_merge_win.cuh): the A share of consecutive subtiles jumps
+    between 0 and 1, drifts, or differs between the two runs of a group."""
+    h = si.uniform_u32(n, seed)
+    i = np.arange(n, dtype=np.uint64)
+    if kind == "sawtooth":          # sorted segments of random length
+        seg = np.cumsum(1 + (si.uniform_u32(n // 64 + 2, seed + 1) % 20000)).astype(np.int64)
+        start = np.zeros(n, np.int64)
+        idx = np.searchsorted(seg, np.arange(n), side="right")
+        start[:] = np.concatenate([[0], seg])[idx]
+        return (np.arange(n) - start).astype(np.uint32) * np.uint32(977)
+    if kind == "bands":             # chunks drawn from disjoint key bands
+        band = (i // 3000) % 7
+        return ((band.astype(np.uint32) << np.uint32(28)) | (h >> np.uint32(4))).astype(np.uint32)
+    if kind == "scaled":            # uniform, each 1000-chunk scaled differently
+        f = si.uniform_u32(n // 1000 + 1, seed + 2)[i // 1000] >> np.uint32(24)
+        return ((h >> np.uint32(8)) * (f + np.uint32(1))).astype(np.uint32)
+    if kind == "nearly_sorted":     # sorted with 1 % random swaps
+        x = np.arange(n, dtype=np.uint32)
+        k = n // 100
+        a = si.uniform_u32(k, seed + 3) % n
+        b = si.uniform_u32(k, seed + 4) % n
+        for p, q in zip(a, b):
+            x[p], x[q] = x[q], x[p]
+        return x
+    raise ValueError(kind)
+
+
+@pytest.mark.parametrize("kind", ["sawtooth", "bands", "scaled", "nearly_sorted"])
+@pytest.mark.parametrize("E,u", [(31, 128), (15, 256), (9, 128), (31, 256), (17, 512)])
+def test_skewed_window_exhaustion(kind, E, u):
+    # the persistent merge pass ends a subtile early when the merge path
+    # leaves a window; parity must hold for every such subtile
+    n = 300000 + 13
+    x = _skewed(kind, n, si.config_seed(6) + E * 7 + u)
+    got = gpu_sort_u32(x, bcf.make_params(E, u, bcf.ALGO_CONFLICT_FREE))
+    np.testing.assert_array_equal(got, oracle.sort_u32(x), err_msg=f"{kind} E={E} u={u}")
+
+
 def test_extreme_keys_and_pads():
     # real UINT32_MAX keys in a ragged last tile must not be confused with pads
     for n in [4097, 100001]:
