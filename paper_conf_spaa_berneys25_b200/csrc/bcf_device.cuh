@@ -273,6 +273,30 @@ __device__ __forceinline__ int lane_split_smem(const uint32_t* __restrict__ sk, 
 // B_i[(k-j-1) mod E]; both at logical base + idx, B reversed behind A.
 // After the gather, items[] is a circular bitonic sequence starting at k.
 // ---------------------------------------------------------------------------
+// rounds J.. of the gather for rho = identity (keys only): shared byte
+// address = (A or B base, + E words when the round wraps) + 4J, the round
+// index folded into the load's immediate offset (one select, one predicated
+// add and the load per round)
+template <int J, int E, bool FULL_TILE>
+__device__ __forceinline__ void gather_rounds(uint32_t (&key)[E], uint32_t sA, uint32_t sB, uint32_t wmask,
+                                              uint32_t maskA, int k, int nB, uint32_t pad) {
+  if constexpr (J < E) {
+    const bool wrap = (wmask >> J) & 1u;
+    const bool isA = (maskA >> J) & 1u;
+    uint32_t p = isA ? sA : sB;
+    if (wrap) p += 4u * E;
+    if constexpr (FULL_TILE) {
+      asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(key[J]) : "r"(p), "n"(4 * J));
+    } else {
+      const int ia = wrap ? J + E - k : J - k;
+      uint32_t v = pad;
+      if (isA || (E - 1 - ia) < nB) asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(p), "n"(4 * J));
+      key[J] = v;
+    }
+    gather_rounds<J + 1, E, FULL_TILE>(key, sA, sB, wmask, maskA, k, nB, pad);
+  }
+}
+
 template <int E, bool PAIRS, bool FULL_TILE>
 __device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restrict__ sk,
                                                         const uint32_t* __restrict__ sv, int base,
@@ -287,6 +311,14 @@ __device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restri
   const int offB = base + S2 - b - E - k;
   const uint32_t m0 = (1u << nA) - 1u;
   const uint32_t maskA = ((m0 << k) | (m0 >> (E - k))) & ((1u << E) - 1u);
+  if constexpr (cgcd(W, E) == 1 && !PAIRS) {
+    // rho = identity: select one of two shared-memory base pointers per
+    // round and fold the round index into the load's immediate offset
+    const uint32_t sA = (uint32_t)__cvta_generic_to_shared(sk) + 4u * (uint32_t)offA;
+    const uint32_t sB = (uint32_t)__cvta_generic_to_shared(sk) + 4u * (uint32_t)offB;
+    gather_rounds<0, E, FULL_TILE>(key, sA, sB, (1u << k) - 1u, maskA, k, nB, pad);
+    return;
+  }
   const int bAn = offA, bAw = offA + E, bBn = offB, bBw = offB + E;
 #pragma unroll
   for (int j = 0; j < E; ++j) {

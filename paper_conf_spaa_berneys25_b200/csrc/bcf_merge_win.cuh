@@ -235,10 +235,33 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
       asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
       args.trace[(size_t)blockIdx.x * 256 + 255] = smid + 1;
     }
+    // bulk store (TMA) of the outputs the consumers staged in stage s (the
+    // 16-byte aligned middle; warp 0 of the consumers writes the <= 7 + 3
+    // edge words).  Issued and waited on by lane 0 (bulk groups are per thread).
+    auto store_out = [&](int s) {
+      const WinMeta M = meta[s];
+      const int qlo = M.desc ? T - M.cnt : 0, qhi = M.desc ? T : M.cnt;
+      const int w0 = M.cout + qlo, w1 = M.cout + qhi;
+      int ilo = align_up4(w0), ihi = align_dn4(w1);
+      if (lane == 0) {
+        if (ihi > ilo)
+          tma::bulk_s2g(args.dst_k + (M.c0 - M.cout) + ilo, stage(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
+        tma::bulk_commit();
+      }
+    };
+
     load_window(0);
     if (lane == 0) BCF_TRACE_AT(128 + 2);
     for (int i = 0;; ++i) {
       const int s = i % S;
+      const int s1 = (i + 1) % S;
+      if (i >= 1) {
+        // subtile i-1's outputs are staged in s1: stream them out while the
+        // consumers search subtile i's split
+        tma::mbar_wait(&empty_bar[s1], (uint32_t)((i - 1) / S) & 1);
+        if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 3);
+        store_out(s1);
+      }
       // subtile i's own end split, found by its consumers
       tma::mbar_wait(&split_bar[s], (uint32_t)(i / S) & 1);
       if (lane == 0 && i < 7) BCF_TRACE_AT(128 + 4 * i + 1);
@@ -260,16 +283,17 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
           shareA = (grp.na + grp.nb) > 0 ? (int)((grp.na << 16) / (grp.na + grp.nb)) : 32768;
         }
       }
-      const int s1 = (i + 1) % S;
-      if (i >= 1) {
-        // stage s1 held subtile i-1: its consumers must have copied it out
-        tma::mbar_wait(&empty_bar[s1], (uint32_t)((i - 1) / S) & 1);
-        if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 3);
-      }
       if (!more) {
         post_exit(s1);
+        // the last subtile: stream its outputs, then drain every bulk store
+        tma::mbar_wait(&empty_bar[s], (uint32_t)(i / S) & 1);
+        store_out(s);
+        if (lane == 0) tma::bulk_wait_all();
+        __syncwarp();
         break;
       }
+      if (lane == 0) tma::bulk_wait_read_all();  // stage s1's store has read it
+      __syncwarp();
       load_window(s1);
       if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 2);
     }
@@ -358,31 +382,26 @@ __global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, 
 #pragma unroll
       for (int q = 0; q < E; ++q) ok[D + q] = key[q];
     }
+    tma::fence_proxy_async_smem();  // the producer's bulk store reads these words
     tma::named_bar_sync(1, U);
     if (tid == 0 && i < 31) BCF_TRACE_AT(4 + 4 * i);
-    // copy-out: the subtile's outputs sit at stage words [w0, w1), stage word
-    // w belongs at global word g0 + w and both are 16-byte aligned for w = 0
-    // (mod 4): vectorised conflict-free LDS.128 / coalesced STG.128, plus at
-    // most 3 + 3 edge words.
-    {
+    // the producer streams the 16-byte aligned middle of the outputs (stage
+    // word w belongs at global word g0 + w, both aligned for w = 0 mod 4);
+    // warp 0 writes the head/tail edge words, then hands the stage back
+    if (warp == 0) {
       const int qlo = M.desc ? T - cnt : 0;
       const int qhi = M.desc ? T : cnt;
       const int w0 = M.cout + qlo, w1 = M.cout + qhi;
       int ilo = align_up4(w0), ihi = align_dn4(w1);
-      if (ihi < ilo) ilo = ihi = w1;
+      if (ihi <= ilo) ilo = ihi = w1;
       const uint32_t* sb = stage(s);
       uint32_t* gb = args.dst_k + (M.c0 - M.cout);
-#pragma unroll
-      for (int r2 = 0; r2 < (T + 4 * U - 1) / (4 * U) + 1; ++r2) {
-        const int v = ilo + 4 * (tid + r2 * U);
-        if (v < ihi) *reinterpret_cast<uint4*>(gb + v) = *reinterpret_cast<const uint4*>(sb + v);
-      }
-      const int nh = ilo - w0;
-      if (tid < nh) gb[w0 + tid] = sb[w0 + tid];
-      else if (tid >= 32 && tid - 32 < w1 - ihi) gb[ihi + tid - 32] = sb[ihi + tid - 32];
+      const int nh = ilo - w0, nt = w1 - ihi;  // <= 7, <= 3
+      if (lane < nh) gb[w0 + lane] = sb[w0 + lane];
+      else if (lane >= 8 && lane - 8 < nt) gb[ihi + lane - 8] = sb[ihi + lane - 8];
+      __syncwarp();
+      if (lane == 0) tma::mbar_arrive(&empty_bar[s]);
     }
-    tma::named_bar_sync(1, U);  // stage reads done: hand it back to the producer
-    if (tid == 0) tma::mbar_arrive(&empty_bar[s]);
     if (tid == 0 && i < 31) BCF_TRACE_AT(3 + 4 * i);
   }
 }
