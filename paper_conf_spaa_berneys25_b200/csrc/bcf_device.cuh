@@ -149,6 +149,30 @@ __device__ __forceinline__ int warp_origin_smem(const uint32_t* __restrict__ sk,
   int lo = D - NB;
   if (lo < 0) lo = 0;
   int hi = D < NA ? D : NA;
+  if constexpr (cgcd(W, E) == 1) {
+    // rho = identity: any odd stride puts the 32 probes of one load in 32
+    // distinct banks, so each round tests 64 candidates (two loads per side):
+    // a range of 64^2 = 4096 takes two rounds
+    while (hi > lo) {
+      const int cnt = hi - lo;
+      const int s = ((cnt + 63) >> 6) | 1;
+      // candidate i at lo + (i+1)s - 1: load 1 tests i = lane, load 2 i = lane + 32
+      const int q0 = lo + (lane + 1) * s - 1;       // candidate lane
+      const int q1 = lo + (lane + 33) * s - 1;      // candidate lane + 32
+      bool p0 = false, p1 = false;
+      if (q0 < hi) p0 = !(sk[bofs + q0] < sk[base + q0]);
+      if (q1 < hi) p1 = !(sk[bofs + q1] < sk[base + q1]);
+      const unsigned b0 = __ballot_sync(FULL, p0), b1 = __ballot_sync(FULL, p1);
+      const int c = __popc(b0) + __popc(b1);  // monotone: the first c candidates hold
+      const int nlo = lo + c * s;
+      int nhi = lo + (c + 1) * s - 1;
+      if (nhi > hi) nhi = hi;
+      lo = nlo;
+      hi = nhi;
+      if (s == 1) break;
+    }
+    return lo;
+  }
   while (hi - lo > E) {
     const int cnt = hi - lo;
     // stride s = f*E with f odd and 32*s >= cnt: the 32 probes are = const

@@ -119,10 +119,13 @@ __device__ __forceinline__ long long merge_path_warp_global_bounded(const RunVie
   return lo;
 }
 
-// Bracketed merge path that first tests the 64 candidates around a guess
-// (the proportional split of the remaining elements): for random keys the
-// answer lies within +-32 of it with high probability (one round of global
-// latency); otherwise the 64-ary search continues on the reduced bracket.
+// Bracketed merge path that first tests 64 candidates around a guess (the
+// proportional split of the remaining elements), spaced by s1 ~ sqrt(D)/16:
+// for random keys a(D) deviates from the guess by O(sqrt(D)), so it lies
+// inside the probed bracket (+-32 s1, about 8 standard deviations) and a
+// second round at stride 1 (s1 <= 64) finishes the search: two rounds of
+// global-memory latency.  Otherwise the 64-ary search continues on the
+// reduced bracket.
 __device__ __forceinline__ long long merge_path_warp_global_guess(const RunView& A, const RunView& B,
                                                                   long long D, long long lo, long long hi,
                                                                   long long guess, int lane) {
@@ -132,21 +135,30 @@ __device__ __forceinline__ long long merge_path_warp_global_guess(const RunView&
   long long h2 = D < A.len ? D : A.len;
   if (hi > h2) hi = h2;
   if (hi <= lo) return lo;
-  long long L = guess - 32;
-  if (L > hi - 64) L = hi - 64;
+  long long s1 = (long long)sqrtf((float)(D < 1 ? 1 : D)) / 16;
+  if (s1 < 1) s1 = 1;
+  if (s1 > 64) s1 = 64;
+  // probes m_i = L + (i+1) s1 - 1, i = 0..63 (lane tests i = 2 lane, 2 lane + 1)
+  long long L = guess - 32 * s1;
+  if (L > hi - 64 * s1) L = hi - 64 * s1;
   if (L < lo) L = lo;
-  const long long m0 = L + 2 * lane, m1 = m0 + 1;
+  const long long m0 = L + (2 * lane + 1) * s1 - 1, m1 = m0 + s1;
   uint32_t a0 = 0, b0 = 0, a1 = 0, b1 = 0;
   if (m0 < hi) { a0 = A.ld(m0); b0 = B.ld(D - 1 - m0); }
   if (m1 < hi) { a1 = A.ld(m1); b1 = B.ld(D - 1 - m1); }
   const bool p0 = m0 < hi && !(b0 < a0);
   const bool p1 = m1 < hi && !(b1 < a1);
-  const int c = __popc(__ballot_sync(FULL, p0)) + __popc(__ballot_sync(FULL, p1));
-  long long act = hi - L;
-  if (act > 64) act = 64;
-  if (c > 0 && c < act) return L + c;                 // exact: Q(L+c-1) true, Q(L+c) false
-  if (c == 0) return L == lo ? lo : merge_path_warp_global_bounded(A, B, D, lo, L, lane);
-  return L + c == hi ? hi : merge_path_warp_global_bounded(A, B, D, L + c, hi, lane);
+  const unsigned bal0 = __ballot_sync(FULL, p0), bal1 = __ballot_sync(FULL, p1);
+  const int c = __popc(bal0) + __popc(bal1);  // Q true for the first c probes
+  // answer in [L + c s1, L + (c+1) s1 - 1] when probe c exists and is false
+  long long nlo = L + (long long)c * s1;
+  long long nhi = L + (long long)(c + 1) * s1 - 1;
+  if (nhi > hi) nhi = hi;
+  if (c == 0) return L == lo ? (s1 == 1 ? lo : merge_path_warp_global_bounded(A, B, D, lo, L + s1 - 1, lane))
+                             : merge_path_warp_global_bounded(A, B, D, lo, L + s1 - 1, lane);
+  if (c == 64) return merge_path_warp_global_bounded(A, B, D, L + 64 * s1, hi, lane);
+  if (s1 == 1 || nlo >= nhi) return nlo;
+  return merge_path_warp_global_bounded(A, B, D, nlo, nhi, lane);
 }
 
 template <int E, int U, bool PAIRS>

@@ -74,8 +74,14 @@ __device__ __forceinline__ int warp_prefix_count(int n, P pred, int lane) {
   return lo;
 }
 
+// resident CTAs per SM the kernel is built for (5 at u = 128)
+template <int U>
+__host__ __device__ constexpr int win_min_blocks() {
+  return U <= 128 ? 5 : (U <= 256 ? 2 : 1);
+}
+
 template <int E, int U>
-__global__ void __launch_bounds__(U + 32) merge_pass_win_kernel(MergeArgs args, long long tiles,
+__global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_kernel(MergeArgs args, long long tiles,
                                                                 long long per_cta) {
   constexpr int T = U * E;
   constexpr int S2 = win_span<E, U>();
