@@ -142,6 +142,68 @@ def cpu_oracle_rate(n_sample: int, reps: int, kinds, E, u):
     return total_keys / total_s, total_s
 
 
+def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
+    """BASELINE configs[2]: 2^28 f32 keys and 2^26 u32 key-value pairs (stable),
+    each timed like the headline (device-resident inputs, L2 flushed between
+    steps, CUDA events on the launch stream), plus the merge pass's achieved
+    HBM bandwidth (f32: 8 B/key, pairs: 16 B/pair per pass)."""
+    import torch
+
+    res = {}
+    legs = [
+        ("f32_2^28", 1 << 28, 8),
+        ("pairs_u32_2^26", 1 << 26, 16),
+    ]
+    for name, n, bpk in legs:
+        if name.startswith("f32"):
+            x = si.uniform_f32_torch(n, si.config_seed(3), dev)
+            out = torch.empty_like(x)
+            run = lambda: bcf.sort(x, out=out, params=params, temp=temp)  # noqa: E731
+            workload = "2^28 float32 keys, uniform [0,1) (24-bit mantissa grid), IEEE totalOrder"
+        else:
+            k = si.dup_u32_torch(n, si.config_seed(4), dev)
+            v = si.iota_u32_torch(n, dev)
+            ko, vo = torch.empty_like(k), torch.empty_like(v)
+            prm = bcf.default_pairs_params()  # pairs default (17, 256)
+            run = lambda: bcf.sort_pairs(k, v, ko, vo, params=prm, temp=temp)  # noqa: E731
+            workload = "2^26 uint32 (key & 0xFFFF, heavy duplicates) + uint32 value (index) pairs, stable"
+        if name.startswith("f32"):
+            prm = params
+        temp = bcf.temp_buffer(n, prm, pairs=name.startswith("pairs"), device=dev)
+        for _ in range(3):
+            run()
+        torch.cuda.synchronize()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+        for i in range(steps):
+            flush.fill_(i)
+            ev[i][0].record(stream)
+            run()
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        ms = sum(s.elapsed_time(e) for s, e in ev) / steps
+        bcf.profile_enable(True)
+        for i in range(3):
+            flush.fill_(i)
+            run()
+        torch.cuda.synchronize()
+        bcf.profile_enable(False)
+        prof = bcf.profile_collect()
+        mp = prof.get("merge_pass", {"launches": 0, "total_ms": 0.0})
+        bs = prof.get("block_sort", {"launches": 0, "total_ms": 0.0})
+        avg = mp["total_ms"] / max(1, mp["launches"])
+        res[name] = {"workload": workload, "n": n, "E": prm.items_per_thread, "u": prm.block_threads,
+                     "value": n / (ms / 1e3),
+                     "unit": "pairs/s" if name.startswith("pairs") else "keys/s", "ms_per_sort": ms,
+                     "merge_pass": {"launches_per_sort": mp["launches"] // 3, "avg_ms": avg,
+                                    "achieved_gbs": bpk * n / (avg / 1e3) / 1e9 if avg else None,
+                                    "frac_of_hbm": (bpk * n / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
+                                    "bytes_per_launch": bpk * n},
+                     "block_sort_ms": bs["total_ms"] / max(1, bs["launches"])}
+        del run, temp
+        torch.cuda.empty_cache()
+    return res
+
+
 def run_reference(a):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -365,6 +427,8 @@ def main():
                               "worst_keys_per_s": len(w_) * n / (sum(w_) / 1e3),
                               "worst_over_random_time": statistics.mean(w_) / statistics.mean(r_)}
         line["contrast"] = contrast
+
+        line["configs_extra"] = extra_configs(bcf, dev, stream, flush, params, peaks)
 
         rate, secs = cpu_oracle_rate(n, 3, ["random", "worst", "random"], E, u)
         line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",

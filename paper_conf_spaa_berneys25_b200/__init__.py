@@ -32,7 +32,7 @@ ALGO_BASELINE = 1
 
 # every symbol include/bcf.h declares
 EXPORTED_SYMBOLS = [
-    "bcf_default_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
+    "bcf_default_params", "bcf_default_pairs_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
     "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
     "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
@@ -69,6 +69,8 @@ def lib():
     P = ctypes.POINTER
     L.bcf_default_params.argtypes = [P(Params)]
     L.bcf_default_params.restype = None
+    L.bcf_default_pairs_params.argtypes = [P(Params)]
+    L.bcf_default_pairs_params.restype = None
     for name in ("bcf_sort_u32", "bcf_sort_f32"):
         f = getattr(L, name)
         f.argtypes = [vp, vp, u64, vp, P(sz), P(Params), vp]
@@ -110,6 +112,12 @@ def default_params() -> Params:
     return p
 
 
+def default_pairs_params() -> Params:
+    p = Params()
+    lib().bcf_default_pairs_params(ctypes.byref(p))
+    return p
+
+
 def make_params(E: int = 0, u: int = 0, algo: int = ALGO_CONFLICT_FREE) -> Params:
     return Params(E, u, algo)
 
@@ -138,6 +146,19 @@ def _stream(t):
 def _temp(nbytes: int, device):
     torch = _torch()
     return torch.empty(max(1, int(nbytes)), dtype=torch.uint8, device=device)
+
+
+def temp_buffer(n: int, params: Params | None = None, pairs: bool = False, device="cuda"):
+    """Temp storage for a sort of n keys (or pairs) with `params`, sized by the
+    library's CUB-style query (d_temp = NULL)."""
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    L = lib()
+    if pairs:
+        _check(L.bcf_sort_pairs_u32(None, None, None, None, n, None, ctypes.byref(tb), pp, None), "temp query")
+    else:
+        _check(L.bcf_sort_u32(None, None, n, None, ctypes.byref(tb), pp, None), "temp query")
+    return _temp(tb.value, device)
 
 
 def sort(keys, out=None, params: Params | None = None, temp=None):

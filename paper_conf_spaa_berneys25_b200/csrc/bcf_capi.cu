@@ -50,6 +50,11 @@ LaunchTable& launch_table() {
 // keeps the tile (3968 keys) and the per-thread registers within budget.
 static constexpr int DEFAULT_E = 31;
 static constexpr int DEFAULT_U = 128;
+// Pairs carry a value and a tag per register: E = 31 spills the register
+// budget, (17, 256) is the measured best of the pairs sweep at 2^26
+// (profiles/r01_pairs_sweep_2p26.txt: 12.1 G pairs/s vs 7.1 at (31, 128)).
+static constexpr int DEFAULT_E_PAIRS = 17;
+static constexpr int DEFAULT_U_PAIRS = 256;
 
 // ---------------------------------------------------------------------------
 // errors, profiler, launch accounting
@@ -105,9 +110,9 @@ struct Params {
   int E, U, algo;
 };
 
-static bcf_status resolve(const bcf_params* p, Params& out) {
-  out.E = (p && p->items_per_thread) ? p->items_per_thread : DEFAULT_E;
-  out.U = (p && p->block_threads) ? p->block_threads : DEFAULT_U;
+static bcf_status resolve(const bcf_params* p, Params& out, bool pairs) {
+  out.E = (p && p->items_per_thread) ? p->items_per_thread : (pairs ? DEFAULT_E_PAIRS : DEFAULT_E);
+  out.U = (p && p->block_threads) ? p->block_threads : (pairs ? DEFAULT_U_PAIRS : DEFAULT_U);
   out.algo = p ? p->algo : BCF_ALGO_CONFLICT_FREE;
   if (out.algo != BCF_ALGO_CONFLICT_FREE && out.algo != BCF_ALGO_BASELINE) return BCF_ERROR_INVALID_VALUE;
   if (out.E < E_MIN || out.E > E_MAX || (out.E > 17 && out.E != 31) || u_index(out.U) < 0)
@@ -154,7 +159,7 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
                             cudaStream_t s, bool f32, bool pairs) {
   if (!temp_bytes) return BCF_ERROR_INVALID_VALUE;
   Params p;
-  bcf_status st = resolve(pp, p);
+  bcf_status st = resolve(pp, p, pairs);
   if (st != BCF_SUCCESS) return st;
   if (pairs && p.algo == BCF_ALGO_BASELINE) return BCF_ERROR_UNSUPPORTED;
   // two ping-pong buffers X, Y (256-B aligned, 64 words of slack for the
@@ -241,6 +246,13 @@ void bcf_default_params(bcf_params* p) {
   p->algo = BCF_ALGO_CONFLICT_FREE;
 }
 
+void bcf_default_pairs_params(bcf_params* p) {
+  if (!p) return;
+  p->items_per_thread = DEFAULT_E_PAIRS;
+  p->block_threads = DEFAULT_U_PAIRS;
+  p->algo = BCF_ALGO_CONFLICT_FREE;
+}
+
 bcf_status bcf_sort_u32(const uint32_t* d_in, uint32_t* d_out, uint64_t n, void* d_temp,
                         size_t* temp_bytes, const bcf_params* p, void* stream) {
   return sort_impl(d_in, d_out, nullptr, nullptr, n, d_temp, temp_bytes, p, (cudaStream_t)stream, false,
@@ -310,11 +322,11 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   // Pairwise merge tree over the runs in run order (run 2g is A, 2g+1 is B,
   // ties to A = the lower run), table mode of the CF merge-pass kernel.
   if (!temp_bytes || nruns < 0 || (nruns > 0 && !h_run_offsets)) return BCF_ERROR_INVALID_VALUE;
+  const bool pairs = d_run_vals != nullptr;
   Params p;
-  bcf_status st = resolve(pp, p);
+  bcf_status st = resolve(pp, p, pairs);
   if (st != BCF_SUCCESS) return st;
   if (p.algo != BCF_ALGO_CONFLICT_FREE) return BCF_ERROR_UNSUPPORTED;
-  const bool pairs = d_run_vals != nullptr;
   const uint64_t n = nruns > 0 ? h_run_offsets[nruns] : 0;
   for (int r = 0; r < nruns; ++r)
     if (h_run_offsets[r + 1] < h_run_offsets[r] || h_run_offsets[0] != 0) return BCF_ERROR_INVALID_VALUE;

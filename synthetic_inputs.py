@@ -159,3 +159,23 @@ def uniform_u32_torch(n: int, seed: int, device, lo: int = 0):
     h = splitmix64_torch(seed, lo, lo + n, device)
     hi = _lsr(h, 32)
     return (hi - ((hi >= (1 << 31)).to(torch.int64) << 32)).to(torch.int32)
+
+
+def uniform_f32_torch(n: int, seed: int, device, lo: int = 0):
+    """Same values as uniform_f32 (exact: 24-bit integers times 2^-24), as a float32 tensor."""
+    import torch
+
+    h = splitmix64_torch(seed, lo, lo + n, device)
+    return _lsr(h, 40).to(torch.float32) * (2.0 ** -24)
+
+
+def dup_u32_torch(n: int, seed: int, device, lo: int = 0, mask: int = 0xFFFF):
+    """Same values as dup_u32, as an int32 tensor."""
+    return uniform_u32_torch(n, seed, device, lo) & mask
+
+
+def iota_u32_torch(n: int, device, lo: int = 0):
+    """Same values as iota_u32 (for n + lo <= 2^31), as an int32 tensor."""
+    import torch
+
+    return torch.arange(lo, lo + n, dtype=torch.int64, device=device).to(torch.int32)

@@ -52,6 +52,8 @@ def test_default_params():
     assert 7 <= p.items_per_thread <= 17 or p.items_per_thread == 31
     assert p.block_threads in (128, 256, 512)
     assert p.algo == bcf.ALGO_CONFLICT_FREE
+    q = bcf.default_pairs_params()
+    assert (q.items_per_thread, q.block_threads, q.algo) == (17, 256, bcf.ALGO_CONFLICT_FREE)
 
 
 def _query(fn, n, params=None, pairs=False):

@@ -9,6 +9,13 @@
 //   case 4  mbarrier.try_wait spin by 128 threads on one barrier (thread 128 arrives late)
 //   case 5  LDS.128 (uint4) stride-1 loads by 128 threads (4 wavefronts per instruction)
 //   case 6  all-thread broadcast read of a 48-byte struct (the merge pass's WinMeta)
+//   case 7  conflict-free stride-1 LDS by warps 0-3 WHILE thread 128 streams bulk
+//           global->shared copies into another smem region (the merge pass's overlap)
+//   case 8  conflict-free stride-1 LDS by warps 0-3 WHILE warp 4 streams LDG (L1 fills)
+//   case 9  stride-31 STS by warps 0-3 (the merge pass's output staging), alone
+//   case 10 stride-31 STS by warps 0-3 WHILE thread 128 streams bulk shared->global
+//   case 11 stride-1 LDS by warps 0-3 WHILE thread 128 streams bulk shared->global
+//   case 12 stride-31 STS by warps 0-3 WHILE thread 128 streams bulk global->shared
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -I<csrc> tools/ncu_calib_tma.cu
 #include <cstdint>
 #include <cstdio>
@@ -32,7 +39,7 @@ extern "C" __global__ void __launch_bounds__(160) calib_tma_kernel(uint32_t* gin
   uint32_t* s = reinterpret_cast<uint32_t*>(sm + ((which == 1 || which == 3) ? 16 : 0));
   if (tid == 0) tma::mbar_init(&bar, 1);
   if (tid < 12) reinterpret_cast<int*>(&meta)[tid] = tid;
-  for (int i = tid; i < BYTES / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(sm)[i] = i;
+  for (int i = tid; i < 2 * BYTES / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(sm)[i] = i;
   tma::fence_proxy_async_smem();
   __syncthreads();
   const uint32_t* src = gin + (size_t)blockIdx.x * (BYTES / 4);
@@ -66,6 +73,46 @@ extern "C" __global__ void __launch_bounds__(160) calib_tma_kernel(uint32_t* gin
         const uint4 v = reinterpret_cast<const uint4*>(sm)[(tid + it) & 1023];
         acc += v.x ^ v.y ^ v.z ^ v.w;
       }
+    } else if (which >= 9) {
+      if (tid < 128) {
+        uint32_t* x = reinterpret_cast<uint32_t*>(sm + BYTES);
+        if (which == 11) {
+#pragma unroll 4
+          for (int q = 0; q < 64; ++q) acc += x[(tid + 32 * q + it) & 4095];
+        } else {
+          // thread t writes words 31 t + q (q = 0..30): a round set per q
+#pragma unroll 4
+          for (int q = 0; q < 31; ++q) x[(31 * tid + q + it) & 4095] = q + it;
+        }
+      } else if (tid == 128 && which != 9) {
+        if (which == 12) {
+          tma::mbar_expect_tx(&bar, BYTES);
+          tma::bulk_g2s(sm, src, BYTES, &bar);
+          tma::mbar_arrive(&bar);
+          tma::mbar_wait(&bar, it & 1);
+        } else {
+          tma::bulk_s2g(dst, sm, BYTES);
+          tma::bulk_commit();
+          tma::bulk_wait_all();
+        }
+      }
+    } else if (which == 7 || which == 8) {
+      if (tid < 128) {
+        const uint32_t* x = reinterpret_cast<const uint32_t*>(sm + BYTES);
+#pragma unroll 4
+        for (int q = 0; q < 64; ++q) acc += x[(tid + 32 * q + it) & 4095];
+      } else if (which == 7) {
+        if (tid == 128) {
+          tma::mbar_expect_tx(&bar, BYTES);
+          tma::bulk_g2s(sm, src, BYTES, &bar);
+          tma::mbar_arrive(&bar);
+          tma::mbar_wait(&bar, it & 1);
+        }
+      } else {
+        const uint32_t* g = src;
+#pragma unroll 4
+        for (int q = 0; q < BYTES / 4 / 32; ++q) acc += __ldg(g + (tid - 128) + 32 * q);
+      }
     } else {
       Meta12 m = meta;
       acc += (uint32_t)m.c0 + m.a[(it + tid) % 10];
@@ -82,9 +129,9 @@ int main() {
   cudaMalloc(&in, words * 4);
   cudaMalloc(&out, words * 4);
   cudaMemset(in, 1, words * 4);
-  cudaFuncSetAttribute(calib_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, BYTES + 128);
-  for (int which = 0; which <= 6; ++which) {
-    calib_tma_kernel<<<148, 160, BYTES + 128>>>(in, out, which, 64);
+  cudaFuncSetAttribute(calib_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * BYTES + 128);
+  for (int which = 0; which <= 12; ++which) {
+    calib_tma_kernel<<<148, 160, 2 * BYTES + 128>>>(in, out, which, 64);
     cudaError_t e = cudaDeviceSynchronize();
     printf("case %d: %s\n", which, cudaGetErrorString(e));
   }
