@@ -86,6 +86,21 @@ bcf_status bcf_sort_u32(const uint32_t* d_in, uint32_t* d_out, uint64_t n, void*
 bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_temp,
                         size_t* temp_bytes, const bcf_params* p, void* stream);
 
+/* End-to-end sort of nbatch independent HOST arrays of n u32 keys each:
+   h_in[i] -> (H2D) -> bcf_sort_u32 -> (D2H) -> h_out[i] (h_out[i] may equal
+   h_in[i]; the h_in/h_out pointer arrays are host arrays).  Two device slots:
+   the H2D copy of batch i+1 and the D2H copy of batch i-1 run on the
+   library's own copy streams while batch i sorts on `stream`, so the
+   throughput is bounded by max(H2D, sort, D2H) per batch.  Host buffers
+   should be pinned (cudaHostAlloc / torch pin_memory) for the copies to be
+   asynchronous; pageable memory is correct but serialises.  Temp (CUB-style
+   query with d_temp = NULL): 4 n keys + the sort's temp.  Stream-ordered:
+   the work starts after the work already queued on `stream`, and `stream`
+   completes after the last read-back (synchronise it before reading h_out). */
+bcf_status bcf_sort_u32_host_batch(const uint32_t* const* h_in, uint32_t* const* h_out, int32_t nbatch,
+                                   uint64_t n, void* d_temp, size_t* temp_bytes, const bcf_params* p,
+                                   void* stream);
+
 /* Stable sort of (key, value) pairs by u32 key; values (u32) follow their
    keys; equal keys keep their input order.  Temp: n keys + n values.
    BCF_ALGO_BASELINE is not supported for pairs (BCF_ERROR_UNSUPPORTED). */

@@ -33,7 +33,7 @@ ALGO_BASELINE = 1
 # every symbol include/bcf.h declares
 EXPORTED_SYMBOLS = [
     "bcf_default_params", "bcf_default_pairs_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
-    "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
+    "bcf_sort_u32_host_batch", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
     "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
 ]
@@ -75,6 +75,8 @@ def lib():
         f = getattr(L, name)
         f.argtypes = [vp, vp, u64, vp, P(sz), P(Params), vp]
         f.restype = ctypes.c_int
+    L.bcf_sort_u32_host_batch.argtypes = [P(vp), P(vp), i32, u64, vp, P(sz), P(Params), vp]
+    L.bcf_sort_u32_host_batch.restype = ctypes.c_int
     L.bcf_sort_pairs_u32.argtypes = [vp, vp, vp, vp, u64, vp, P(sz), P(Params), vp]
     L.bcf_sort_pairs_u32.restype = ctypes.c_int
     L.bcf_worst_case_u32.argtypes = [vp, u64, i32, i32, u64, vp]
@@ -205,6 +207,40 @@ def sort_pairs(keys, values, keys_out=None, values_out=None, params: Params | No
                                     values_out.data_ptr(), n, temp.data_ptr(), ctypes.byref(tb), pp,
                                     _stream(keys)), "bcf_sort_pairs_u32")
     return keys_out, values_out
+
+
+def sort_host_batch(h_in, h_out, params: Params | None = None, temp=None, device="cuda"):
+    """End-to-end sort of a batch of host (CPU) arrays of equal length n
+    (bcf_sort_u32_host_batch): H2D, sort and D2H of consecutive arrays overlap.
+    h_in / h_out: sequences of 1-D CPU tensors (pinned for async copies) of
+    4-byte elements, sorted as u32 bit patterns.  Returns after the library's
+    work is queued on the current stream of `device`; synchronise before
+    reading h_out."""
+    torch = _torch()
+    if len(h_in) != len(h_out):
+        raise BcfError("h_in and h_out differ in length")
+    n = h_in[0].numel() if len(h_in) else 0
+    for t in list(h_in) + list(h_out):
+        if not isinstance(t, torch.Tensor) or t.is_cuda or t.element_size() != 4 or not t.is_contiguous() \
+                or t.numel() != n:
+            raise BcfError("h_in/h_out must be contiguous CPU tensors of n 4-byte elements")
+    dev = torch.device(device)
+    if dev.index is None:
+        dev = torch.device("cuda", torch.cuda.current_device())
+    L = lib()
+    pp = ctypes.byref(params) if params is not None else None
+    tb = ctypes.c_size_t(0)
+    _check(L.bcf_sort_u32_host_batch(None, None, len(h_in), n, None, ctypes.byref(tb), pp, None), "temp query")
+    if temp is None or temp.numel() < tb.value:
+        temp = _temp(tb.value, dev)
+    tb = ctypes.c_size_t(temp.numel())
+    ins = (ctypes.c_void_p * max(1, len(h_in)))(*[t.data_ptr() for t in h_in])
+    outs = (ctypes.c_void_p * max(1, len(h_out)))(*[t.data_ptr() for t in h_out])
+    with torch.cuda.device(dev):
+        _check(L.bcf_sort_u32_host_batch(ins, outs, len(h_in), n, temp.data_ptr(), ctypes.byref(tb), pp,
+                                         ctypes.c_void_p(torch.cuda.current_stream(dev).cuda_stream)),
+               "bcf_sort_u32_host_batch")
+    return h_out
 
 
 def worst_case(n: int, E: int, u: int, seed: int = 0, device="cuda"):

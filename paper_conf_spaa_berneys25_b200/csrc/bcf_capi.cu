@@ -211,6 +211,97 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
 }
 
 // ---------------------------------------------------------------------------
+// host-buffer batches: H2D of batch i+1 and D2H of batch i-1 overlap the sort
+// of batch i (copy engines run both directions at once); two device slots
+// ---------------------------------------------------------------------------
+struct CopyStreams {
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+};
+
+static cudaError_t copy_streams(CopyStreams& cs) {
+  static std::mutex mu;
+  static CopyStreams per_dev[64];
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lk(mu);
+  CopyStreams& c = per_dev[dev];
+  if (!c.h2d) {
+    e = cudaStreamCreateWithFlags(&c.h2d, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return e;
+    e = cudaStreamCreateWithFlags(&c.d2h, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return e;
+  }
+  cs = c;
+  return cudaSuccess;
+}
+
+static bcf_status host_batch_impl(const uint32_t* const* h_in, uint32_t* const* h_out, int32_t nbatch,
+                                  uint64_t n, void* d_temp, size_t* temp_bytes, const bcf_params* pp,
+                                  cudaStream_t s, bool f32) {
+  if (!temp_bytes || nbatch < 0) return BCF_ERROR_INVALID_VALUE;
+  size_t sort_bytes = 0;
+  bcf_status st = sort_impl(nullptr, nullptr, nullptr, nullptr, n, nullptr, &sort_bytes, pp, s, f32, false);
+  if (st != BCF_SUCCESS) return st;
+  const size_t key_bytes = align_up((size_t)n * sizeof(uint32_t), 256);
+  const size_t need = 256 + 4 * key_bytes + sort_bytes;
+  if (d_temp == nullptr) {
+    *temp_bytes = need;
+    return BCF_SUCCESS;
+  }
+  if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
+  if (nbatch == 0 || n == 0) return BCF_SUCCESS;
+  if (!h_in || !h_out) return BCF_ERROR_INVALID_VALUE;
+  for (int i = 0; i < nbatch; ++i)
+    if (!h_in[i] || !h_out[i]) return BCF_ERROR_INVALID_VALUE;
+  CopyStreams cs;
+  cudaError_t e = copy_streams(cs);
+  if (e != cudaSuccess) return cuda_fail(e);
+  char* tb = (char*)align_up((size_t)d_temp, 256);
+  uint32_t* din[2] = {(uint32_t*)tb, (uint32_t*)(tb + key_bytes)};
+  uint32_t* dout[2] = {(uint32_t*)(tb + 2 * key_bytes), (uint32_t*)(tb + 3 * key_bytes)};
+  void* stemp = tb + 4 * key_bytes;
+  // events: entry (caller-stream order), per slot: input landed, sorted, output read back
+  cudaEvent_t ev[7];
+  for (auto& x : ev) {
+    e = cudaEventCreateWithFlags(&x, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_fail(e);
+  }
+  cudaEvent_t entry = ev[0], in_ok[2] = {ev[1], ev[2]}, sorted[2] = {ev[3], ev[4]}, out_ok[2] = {ev[5], ev[6]};
+  auto chk = [&](cudaError_t x) {
+    if (x != cudaSuccess && e == cudaSuccess) e = x;
+  };
+  chk(cudaEventRecord(entry, s));
+  chk(cudaStreamWaitEvent(cs.h2d, entry, 0));
+  chk(cudaStreamWaitEvent(cs.d2h, entry, 0));
+  const size_t bytes = (size_t)n * sizeof(uint32_t);
+  for (int i = 0; i < nbatch && e == cudaSuccess; ++i) {
+    const int k = i & 1;
+    if (i >= 2) chk(cudaStreamWaitEvent(cs.h2d, sorted[k], 0));  // sort i-2 has read din[k]
+    chk(cudaMemcpyAsync(din[k], h_in[i], bytes, cudaMemcpyHostToDevice, cs.h2d));
+    chk(cudaEventRecord(in_ok[k], cs.h2d));
+    chk(cudaStreamWaitEvent(s, in_ok[k], 0));
+    if (i >= 2) chk(cudaStreamWaitEvent(s, out_ok[k], 0));  // D2H i-2 has read dout[k]
+    if (e != cudaSuccess) break;
+    size_t sb = sort_bytes;
+    st = sort_impl(din[k], dout[k], nullptr, nullptr, n, stemp, &sb, pp, s, f32, false);
+    if (st != BCF_SUCCESS) break;
+    chk(cudaEventRecord(sorted[k], s));
+    chk(cudaStreamWaitEvent(cs.d2h, sorted[k], 0));
+    chk(cudaMemcpyAsync(h_out[i], dout[k], bytes, cudaMemcpyDeviceToHost, cs.d2h));
+    chk(cudaEventRecord(out_ok[k], cs.d2h));
+  }
+  // the caller's stream completes after the last read-back
+  chk(cudaEventRecord(out_ok[0], cs.d2h));
+  chk(cudaStreamWaitEvent(s, out_ok[0], 0));
+  chk(cudaStreamWaitEvent(cs.h2d, out_ok[0], 0));
+  for (auto& x : ev) cudaEventDestroy(x);
+  if (st != BCF_SUCCESS) return st;
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
+// ---------------------------------------------------------------------------
 // distributed helpers
 // ---------------------------------------------------------------------------
 __global__ void split_counts_kernel(const uint32_t* __restrict__ a, unsigned long long n,
@@ -263,6 +354,12 @@ bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_tem
                         const bcf_params* p, void* stream) {
   return sort_impl((const uint32_t*)d_in, (uint32_t*)d_out, nullptr, nullptr, n, d_temp, temp_bytes, p,
                    (cudaStream_t)stream, true, false);
+}
+
+bcf_status bcf_sort_u32_host_batch(const uint32_t* const* h_in, uint32_t* const* h_out, int32_t nbatch,
+                                   uint64_t n, void* d_temp, size_t* temp_bytes, const bcf_params* p,
+                                   void* stream) {
+  return host_batch_impl(h_in, h_out, nbatch, n, d_temp, temp_bytes, p, (cudaStream_t)stream, false);
 }
 
 bcf_status bcf_sort_pairs_u32(const uint32_t* d_keys_in, uint32_t* d_keys_out, const uint32_t* d_vals_in,

@@ -119,3 +119,27 @@ def test_host_worst_case_is_permutation_at_bench_size():
     n = 1 << 22
     x = bcf.worst_case_host(n, 16, 256, 0xB2000001)
     assert np.array_equal(np.sort(x), np.arange(n, dtype=np.uint32))
+
+
+def test_host_batch_query_and_validation():
+    """bcf_sort_u32_host_batch: CUB-style temp query (two device slots of
+    input + output keys plus the sort's own temp) and synchronous argument
+    errors, all without touching a GPU."""
+    L = bcf.lib()
+    for n in [0, 1000, 1 << 24]:
+        tb = ctypes.c_size_t(0)
+        assert L.bcf_sort_u32_host_batch(None, None, 3, n, None, ctypes.byref(tb), None, None) == 0
+        _, sort_tb = _query(L.bcf_sort_u32, n)
+        assert tb.value >= 16 * n + sort_tb
+    tb = ctypes.c_size_t(0)
+    assert L.bcf_sort_u32_host_batch(None, None, -1, 10, None, ctypes.byref(tb), None,
+                                     None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_sort_u32_host_batch(None, None, 1, 10, None, None, None, None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_sort_u32_host_batch(None, None, 1, 10, None, ctypes.byref(tb), ctypes.byref(bcf.make_params(18, 256)),
+                                     None) == bcf.BCF_ERROR_UNSUPPORTED
+    # null host arrays with a real temp pointer: rejected before any copy
+    assert L.bcf_sort_u32_host_batch(None, None, 0, 10, None, ctypes.byref(tb), None, None) == 0
+    need = tb.value
+    tb = ctypes.c_size_t(need)
+    assert L.bcf_sort_u32_host_batch(None, None, 2, 10, ctypes.c_void_p(256), ctypes.byref(tb), None,
+                                     None) == bcf.BCF_ERROR_INVALID_VALUE

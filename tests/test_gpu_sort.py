@@ -248,3 +248,26 @@ def test_full_2p28_f32_properties():
     np.testing.assert_array_equal(
         bcf.sort(torch.from_numpy(x[:m]).to(DEV)).cpu().numpy().view(np.uint32),
         oracle.sort_f32_bits(x[:m].view(np.uint32)))
+
+
+@pytest.mark.parametrize("nbatch,n", [(1, 1), (3, 4097), (5, 100003), (4, 1 << 20)])
+def test_host_batch_parity(nbatch, n):
+    """bcf_sort_u32_host_batch: H2D / sort / D2H pipelined over host arrays
+    (pinned and one pageable), every output against the oracle."""
+    xs = []
+    for i in range(nbatch):
+        seed = si.config_seed(6) + 31 * i + n
+        x = si.uniform_u32(n, seed) if i % 2 == 0 else bcf.worst_case_host(n, 31, 128, seed)
+        xs.append(x)
+    h_in = [torch.from_numpy(x.view(np.int32).copy()) for x in xs]
+    h_in = [t.pin_memory() if i != 1 else t for i, t in enumerate(h_in)]
+    h_out = [torch.empty(n, dtype=torch.int32).pin_memory() for _ in range(nbatch)]
+    bcf.sort_host_batch(h_in, h_out, device=DEV)
+    torch.cuda.synchronize()
+    for i, x in enumerate(xs):
+        np.testing.assert_array_equal(h_out[i].numpy().view(np.uint32), oracle.sort_u32(x), err_msg=f"batch {i}")
+    # in place (h_out[i] is h_in[i])
+    bcf.sort_host_batch(h_in, h_in, device=DEV)
+    torch.cuda.synchronize()
+    for i, x in enumerate(xs):
+        np.testing.assert_array_equal(h_in[i].numpy().view(np.uint32), oracle.sort_u32(x), err_msg=f"in place {i}")

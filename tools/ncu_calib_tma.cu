@@ -16,6 +16,8 @@
 //   case 10 stride-31 STS by warps 0-3 WHILE thread 128 streams bulk shared->global
 //   case 11 stride-1 LDS by warps 0-3 WHILE thread 128 streams bulk shared->global
 //   case 12 stride-31 STS by warps 0-3 WHILE thread 128 streams bulk global->shared
+//   case 13 stride-31 STS by warps 0-3 WHILE warp 4 streams LDG (L1 fills)
+//   case 14 stride-1 LDS by warps 0-3 WHILE warp 4 streams STG
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -I<csrc> tools/ncu_calib_tma.cu
 #include <cstdint>
 #include <cstdio>
@@ -76,7 +78,7 @@ extern "C" __global__ void __launch_bounds__(160) calib_tma_kernel(uint32_t* gin
     } else if (which >= 9) {
       if (tid < 128) {
         uint32_t* x = reinterpret_cast<uint32_t*>(sm + BYTES);
-        if (which == 11) {
+        if (which == 11 || which == 14) {
 #pragma unroll 4
           for (int q = 0; q < 64; ++q) acc += x[(tid + 32 * q + it) & 4095];
         } else {
@@ -84,6 +86,12 @@ extern "C" __global__ void __launch_bounds__(160) calib_tma_kernel(uint32_t* gin
 #pragma unroll 4
           for (int q = 0; q < 31; ++q) x[(31 * tid + q + it) & 4095] = q + it;
         }
+      } else if (which == 13) {
+#pragma unroll 4
+        for (int q = 0; q < BYTES / 4 / 32; ++q) acc += __ldg(src + (tid - 128) + 32 * q);
+      } else if (which == 14) {
+#pragma unroll 4
+        for (int q = 0; q < BYTES / 4 / 32; ++q) dst[(tid - 128) + 32 * q] = q + it;
       } else if (tid == 128 && which != 9) {
         if (which == 12) {
           tma::mbar_expect_tx(&bar, BYTES);
@@ -130,7 +138,7 @@ int main() {
   cudaMalloc(&out, words * 4);
   cudaMemset(in, 1, words * 4);
   cudaFuncSetAttribute(calib_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * BYTES + 128);
-  for (int which = 0; which <= 12; ++which) {
+  for (int which = 0; which <= 14; ++which) {
     calib_tma_kernel<<<148, 160, 2 * BYTES + 128>>>(in, out, which, 64);
     cudaError_t e = cudaDeviceSynchronize();
     printf("case %d: %s\n", which, cudaGetErrorString(e));
