@@ -333,9 +333,9 @@ def main():
     wst = [m for i, m in enumerate(ms) if i % 2 == 1]
 
     peaks, peak_src = measured_peaks()
-    T = E * u
-    tiles = -(-n // T)
-    passes = max(0, (tiles - 1).bit_length())
+    plan = bcf.sort_plan(n, params)
+    T = plan["merge_tile"]
+    passes = plan["merge_passes"]
     roof = None
     mp = prof.get("merge_pass")
     if mp and mp["launches"]:
@@ -361,7 +361,7 @@ def main():
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
         "warmup": max(3, a.warmup), "ms_per_step": total_ms_max / a.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": WORKLOAD, "n": n, "n_per_gpu": n, "E": E, "u": u, "tile": T,
+        "config": {"workload": WORKLOAD, "n": n, "n_per_gpu": n, "E": E, "u": u, "tile": T, "block_sort_tile": plan["block_sort_tile"],
                    "merge_passes": passes, "algo": "conflict_free" if a.algo == 0 else "baseline",
                    "steps_alternate": "random, worst-case (ABAB)",
                    "l2": "flushed between timed steps (256 MiB write, outside the events)",

@@ -86,6 +86,13 @@ bcf_status bcf_sort_u32(const uint32_t* d_in, uint32_t* d_out, uint64_t n, void*
 bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_temp,
                         size_t* temp_bytes, const bcf_params* p, void* stream);
 
+/* The pass plan a sort of n keys (pairs != 0: pairs) with params p runs
+   (host only, no CUDA call): block-sort tile (keys per block-sort CTA; the
+   keys-only CF default (31, 128) sorts tiles of 2u threads), merge-pass tile
+   u*E, and the number of pairwise merge passes ceil(log2(n / block tile)). */
+bcf_status bcf_sort_plan(uint64_t n, const bcf_params* p, int32_t pairs, int64_t* block_sort_tile,
+                         int64_t* merge_tile, int32_t* merge_passes);
+
 /* End-to-end sort of nbatch independent HOST arrays of n u32 keys each:
    h_in[i] -> (H2D) -> bcf_sort_u32 -> (D2H) -> h_out[i] (h_out[i] may equal
    h_in[i]; the h_in/h_out pointer arrays are host arrays).  Two device slots:

@@ -33,7 +33,7 @@ ALGO_BASELINE = 1
 # every symbol include/bcf.h declares
 EXPORTED_SYMBOLS = [
     "bcf_default_params", "bcf_default_pairs_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
-    "bcf_sort_u32_host_batch", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
+    "bcf_sort_u32_host_batch", "bcf_sort_plan", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
     "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
 ]
@@ -75,6 +75,8 @@ def lib():
         f = getattr(L, name)
         f.argtypes = [vp, vp, u64, vp, P(sz), P(Params), vp]
         f.restype = ctypes.c_int
+    L.bcf_sort_plan.argtypes = [u64, P(Params), i32, P(ctypes.c_int64), P(ctypes.c_int64), P(i32)]
+    L.bcf_sort_plan.restype = ctypes.c_int
     L.bcf_sort_u32_host_batch.argtypes = [P(vp), P(vp), i32, u64, vp, P(sz), P(Params), vp]
     L.bcf_sort_u32_host_batch.restype = ctypes.c_int
     L.bcf_sort_pairs_u32.argtypes = [vp, vp, vp, vp, u64, vp, P(sz), P(Params), vp]
@@ -118,6 +120,15 @@ def default_pairs_params() -> Params:
     p = Params()
     lib().bcf_default_pairs_params(ctypes.byref(p))
     return p
+
+
+def sort_plan(n: int, params: Params | None = None, pairs: bool = False) -> dict:
+    """Pass plan of a sort (bcf_sort_plan): block-sort tile, merge tile, passes."""
+    bt, mt, mp = ctypes.c_int64(0), ctypes.c_int64(0), ctypes.c_int32(0)
+    pp = ctypes.byref(params) if params is not None else None
+    _check(lib().bcf_sort_plan(n, pp, 1 if pairs else 0, ctypes.byref(bt), ctypes.byref(mt), ctypes.byref(mp)),
+           "bcf_sort_plan")
+    return {"block_sort_tile": bt.value, "merge_tile": mt.value, "merge_passes": mp.value}
 
 
 def make_params(E: int = 0, u: int = 0, algo: int = ALGO_CONFLICT_FREE) -> Params:

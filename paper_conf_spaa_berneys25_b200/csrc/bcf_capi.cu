@@ -122,6 +122,17 @@ static bcf_status resolve(const bcf_params* p, Params& out, bool pairs) {
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+// threads per block-sort tile (a power-of-two multiple of u; BCF_BS_SAME=1
+// keeps the block sort at u, for A/B measurements)
+static int bs_threads(const Params& p, bool cf, bool pairs) {
+  static const bool same = [] {
+    const char* v = getenv("BCF_BS_SAME");
+    return v && v[0] == '1';
+  }();
+  if (cf && !pairs && p.E == 31 && p.U == 128 && !same) return 256;
+  return p.U;
+}
+
 // BCF_TRACE=<pass>: record a per-CTA timeline of that merge pass (debug)
 static unsigned long long* g_trace = nullptr;
 static const size_t TRACE_WORDS = 1 << 21;
@@ -177,11 +188,21 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
 
   const Variant& var = launch_table().v[p.E][u_index(p.U)][p.algo][pairs ? 1 : 0];
   if (!var.block_sort || !var.merge) return BCF_ERROR_UNSUPPORTED;
-  const long long T = (long long)p.U * p.E;
-  const long long tiles = (long long)((n + T - 1) / T);
-  int P = 0;
-  while ((T << P) < (long long)n) ++P;
   const bool cf = p.algo == BCF_ALGO_CONFLICT_FREE;
+  // Block-sort tile: keys-only CF at E = 31 sorts tiles of 2u threads (its
+  // first five levels run in registers across the warp, so one more shared
+  // level costs less than the merge pass it saves); merge passes keep u.
+  const int Ubs = bs_threads(p, cf, pairs);
+  const Variant& vbs = launch_table().v[p.E][u_index(Ubs)][p.algo][pairs ? 1 : 0];
+  if (!vbs.block_sort) return BCF_ERROR_UNSUPPORTED;
+  const long long T = (long long)p.U * p.E;
+  const long long Tbs = (long long)Ubs * p.E;
+  const long long tiles = (long long)((n + T - 1) / T);
+  const long long tiles_bs = (long long)((n + Tbs - 1) / Tbs);
+  int lg_bs = 0;
+  while ((p.U << lg_bs) < Ubs) ++lg_bs;
+  int P = 0;
+  while ((Tbs << P) < (long long)n) ++P;
   const bool use_tma = cf && var.merge_tma != nullptr && !tma_disabled();
 
   char* tb = (char*)align_up((size_t)d_temp, 256);
@@ -192,14 +213,14 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
 
   SortArgs sa{in_k, in_v, P == 0 ? out_k : X, P == 0 ? out_v : XV, (long long)n, f32 ? 1 : 0,
               (f32 && P == 0) ? 1 : 0, cf ? 1 : 0};
-  cudaError_t e = launch("block_sort", n, s, [&] { return var.block_sort(sa, tiles, s); });
+  cudaError_t e = launch("block_sort", n, s, [&] { return vbs.block_sort(sa, tiles_bs, s); });
   if (e != cudaSuccess) return cuda_fail(e);
   for (int i = 1; i <= P; ++i) {
     uint32_t* sk = (i & 1) ? X : Y;
     uint32_t* sv = (i & 1) ? XV : YV;
     uint32_t* dk = i == P ? out_k : ((i & 1) ? Y : X);
     uint32_t* dv = i == P ? out_v : ((i & 1) ? YV : XV);
-    MergeArgs ma{sk, sv, dk, dv, (long long)n, T << (i - 1), i,
+    MergeArgs ma{sk, sv, dk, dv, (long long)n, Tbs << (i - 1), i + lg_bs,
                  (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0, trace_for_pass(i)};
     if (use_tma)
       e = launch("merge_pass", n, s, [&] { return var.merge_tma(ma, tiles, s); });
@@ -354,6 +375,21 @@ bcf_status bcf_sort_f32(const float* d_in, float* d_out, uint64_t n, void* d_tem
                         const bcf_params* p, void* stream) {
   return sort_impl((const uint32_t*)d_in, (uint32_t*)d_out, nullptr, nullptr, n, d_temp, temp_bytes, p,
                    (cudaStream_t)stream, true, false);
+}
+
+bcf_status bcf_sort_plan(uint64_t n, const bcf_params* pp, int32_t pairs, int64_t* block_sort_tile,
+                         int64_t* merge_tile, int32_t* merge_passes) {
+  Params p;
+  bcf_status st = resolve(pp, p, pairs != 0);
+  if (st != BCF_SUCCESS) return st;
+  const bool cf = p.algo == BCF_ALGO_CONFLICT_FREE;
+  const long long Tbs = (long long)bs_threads(p, cf, pairs != 0) * p.E;
+  int P = 0;
+  while ((Tbs << P) < (long long)n) ++P;
+  if (block_sort_tile) *block_sort_tile = Tbs;
+  if (merge_tile) *merge_tile = (long long)p.U * p.E;
+  if (merge_passes) *merge_passes = P;
+  return BCF_SUCCESS;
 }
 
 bcf_status bcf_sort_u32_host_batch(const uint32_t* const* h_in, uint32_t* const* h_out, int32_t nbatch,

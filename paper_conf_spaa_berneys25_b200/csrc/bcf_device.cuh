@@ -597,6 +597,89 @@ __device__ __forceinline__ void merge_registers(uint32_t (&key)[E], uint32_t (&v
   }
 }
 
+// ---------------------------------------------------------------------------
+// Warp phase of the block sort (keys only, E + 1 = w = 32): the first five
+// merge levels (runs of 1, 2, 4, 8, 16 threads -> runs of one warp) merge
+// registers across lanes with shuffles instead of going through shared
+// memory, so they cannot have bank conflicts at all and cost (L+1) shuffle
+// stages + one in-register bitonic merger at level L instead of a shared
+// scatter / split search / gather.  Every lane holds 32 slots: its E sorted
+// keys and one pad (max key) in slot E.  A level merges the ascending runs of
+// lanes [b, b+h) and [b+h, b+2h) (h = 2^L): a flip stage (slot i of lane t
+// against slot 31-i of lane t ^ (2h-1): the two ascending runs read as one
+// bitonic sequence), half-cleaners across lanes (distance h/2 .. 1), then the
+// 32-slot bitonic merger inside each lane.  Keys only: equal keys are equal
+// bits, so the (unstable) network's order among them is unobservable.
+// After level 4 the warp's 1024 slots are ascending: lanes 0..30 hold its
+// 992 keys (32 each), lane 31 holds the 32 pads.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[W], int lane) {
+#pragma unroll
+  for (int L = 0; L < 5; ++L) {
+    const bool up = (lane >> L) & 1;
+    const int m = (2 << L) - 1;
+#pragma unroll
+    for (int i = 0; i < W / 2; ++i) {
+      const int j = W - 1 - i;
+      const uint32_t pi = __shfl_xor_sync(FULL, k[j], m);
+      const uint32_t pj = __shfl_xor_sync(FULL, k[i], m);
+      k[i] = up ? max(k[i], pi) : min(k[i], pi);
+      k[j] = up ? max(k[j], pj) : min(k[j], pj);
+    }
+#pragma unroll
+    for (int d = L - 1; d >= 0; --d) {
+      const bool hi = (lane >> d) & 1;
+#pragma unroll
+      for (int i = 0; i < W; ++i) {
+        const uint32_t p = __shfl_xor_sync(FULL, k[i], 1 << d);
+        k[i] = hi ? max(k[i], p) : min(k[i], p);
+      }
+    }
+    uint32_t dt[W], dv[W];
+    bitonic_merge_pad<W, false>(k, dt, dv);
+  }
+}
+
+// Conflict-free write of a warp's sorted 992-key run (lanes 0..30 x 32 slots)
+// into the block sort's level-5 layout: the A run (even warp of a merge
+// group) ascending at [gbase, gbase + S), the B run reversed (pi) ending at
+// gbase + 2S (S = 32E).  16-byte stores: in round r lane t writes its quad
+// (r + t) mod 8, so the 8 lanes of each quarter-warp phase hit 8 distinct
+// 16-byte bank groups (the quads are brought into round order by a 3-stage
+// barrel rotation of the registers).
+template <int E>
+__device__ __forceinline__ void warp_run_scatter(uint32_t* __restrict__ sk, const uint32_t (&k)[W], int warp,
+                                                 int lane) {
+  static_assert(E + 1 == W, "warp phase needs E = 31");
+  constexpr int S = W * E;
+  uint32_t r[W];
+#pragma unroll
+  for (int i = 0; i < W; ++i) r[i] = k[i];
+#pragma unroll
+  for (int b = 0; b < 3; ++b) {
+    const bool on = (lane >> b) & 1;
+    uint32_t t[W];
+#pragma unroll
+    for (int i = 0; i < W; ++i) t[i] = on ? r[(i + (4 << b)) % W] : r[i];
+#pragma unroll
+    for (int i = 0; i < W; ++i) r[i] = t[i];
+  }
+  if (lane == W - 1) return;  // the pads
+  const int gbase = (warp >> 1) * 2 * S;
+  const bool isB = warp & 1;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const int qq = (q + lane) & 7;
+    if (isB) {
+      uint4 v = make_uint4(r[4 * q + 3], r[4 * q + 2], r[4 * q + 1], r[4 * q]);
+      *reinterpret_cast<uint4*>(sk + gbase + 2 * S - 4 - W * lane - 4 * qq) = v;
+    } else {
+      uint4 v = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+      *reinterpret_cast<uint4*>(sk + gbase + W * lane + 4 * qq) = v;
+    }
+  }
+}
+
 // f32 <-> order-preserving u32 (IEEE totalOrder, reading c2)
 __device__ __forceinline__ uint32_t f32_encode(uint32_t b) {
   return b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u);

@@ -166,7 +166,7 @@ template <int E, int U, bool PAIRS, bool CF>
 __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
-  extern __shared__ uint32_t smem_dyn[];
+  extern __shared__ __align__(16) uint32_t smem_dyn[];
   uint32_t* sk = smem_dyn;                      // tile_words keys
   uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
   __shared__ int s_org[NW + 1];
@@ -221,9 +221,25 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
   }
   oddeven_sort_pad<E, PAIRS>(key, tag, val);
 
+  // keys only, E = 31: levels 0..4 (runs up to one warp) in registers across
+  // the warp (warp_bitonic_levels), then the warp runs go to shared memory in
+  // the level-5 layout and the CF shared-memory levels continue from l = 5
+  constexpr bool WARP_PHASE = CF && !PAIRS && E + 1 == W && U >= 2 * W;
+  int l_first = 0;
+  if constexpr (WARP_PHASE) {
+    uint32_t k32[W];
+#pragma unroll
+    for (int i = 0; i < E; ++i) k32[i] = key[i];
+    k32[E] = PAD_KEY;
+    warp_bitonic_levels(k32, lane);
+    __syncthreads();  // every thread has finished its blocked read of sk
+    warp_run_scatter<E>(sk, k32, warp, lane);
+    l_first = 5;
+  }
+
   // --- log2(U) merge levels: runs of S = E*2^l, groups of G = 2^(l+1) threads
 #pragma unroll 1
-  for (int l = 0; (1 << l) < U; ++l) {
+  for (int l = l_first; (1 << l) < U; ++l) {
     const int S = E << l;
     const int G = 2 << l;
     const int ir = tid & ((1 << l) - 1);   // index within its run
@@ -231,7 +247,9 @@ __global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
     const int gbase = (run >> 1) * 2 * S;  // group base (logical)
     const bool isB = run & 1;
     __syncthreads();
-    if constexpr (CF) {
+    if (WARP_PHASE && l == 5) {
+      // the warp runs were written by warp_run_scatter
+    } else if constexpr (CF) {
       // conflict-free scatter (fn. 5): B runs are written
       // reversed (pi); in round m B-run lanes write item E-1-m so that every
       // lane writes logical index = m (mod E).  From l = 5 on a run spans
@@ -331,7 +349,7 @@ template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
-  extern __shared__ uint32_t smem_dyn[];
+  extern __shared__ __align__(16) uint32_t smem_dyn[];
   uint32_t* sk = smem_dyn;                      // tile_words keys
   uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
   __shared__ int s_org[NW + 1];

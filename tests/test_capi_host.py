@@ -143,3 +143,18 @@ def test_host_batch_query_and_validation():
     tb = ctypes.c_size_t(need)
     assert L.bcf_sort_u32_host_batch(None, None, 2, 10, ctypes.c_void_p(256), ctypes.byref(tb), None,
                                      None) == bcf.BCF_ERROR_INVALID_VALUE
+
+
+def test_sort_plan():
+    """Pass plan: keys-only CF (31, 128) sorts block tiles of 2u threads; every
+    other configuration (pairs, baseline, other E/u) keeps u; passes =
+    ceil(log2(n / block tile))."""
+    assert bcf.sort_plan(1 << 24) == {"block_sort_tile": 7936, "merge_tile": 3968, "merge_passes": 12}
+    assert bcf.sort_plan(7936)["merge_passes"] == 0
+    assert bcf.sort_plan(7937)["merge_passes"] == 1
+    assert bcf.sort_plan(1 << 24, bcf.make_params(31, 128, bcf.ALGO_BASELINE)) == \
+        {"block_sort_tile": 3968, "merge_tile": 3968, "merge_passes": 13}
+    assert bcf.sort_plan(1 << 26, pairs=True) == {"block_sort_tile": 17 * 256, "merge_tile": 17 * 256,
+                                                  "merge_passes": 14}
+    assert bcf.sort_plan(1 << 24, bcf.make_params(15, 256)) == {"block_sort_tile": 3840, "merge_tile": 3840,
+                                                               "merge_passes": 13}
