@@ -371,6 +371,28 @@ __device__ __forceinline__ void dual_subsequence_gather(const uint32_t* __restri
 // inputs -- a strict total order, so any sorting network yields the stable
 // result.
 // ---------------------------------------------------------------------------
+// Pipe balancing for keys-only compare-exchanges.  min/max run on the ALU
+// pipe (64 lanes/clk/SM, the block sort's bound: ALU pipe ~87 % busy), the
+// FMA pipe is nearly idle.  max(a, b) = a + b - min(a, b) (exact mod 2^32)
+// as two IMADs puts the max on the FMA pipe; the multiplier is read from
+// constant memory so ptxas cannot fold the IMAD back into an ALU IADD3.
+// Networks use this form for 2 of every 3 compare-exchanges (ALU and FMA
+// pipes then carry 4/3 instructions each per exchange instead of 2 + 0).
+static __constant__ uint32_t c_one = 1u;
+
+__device__ __forceinline__ uint32_t imad_u32(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+  return r;
+}
+
+__device__ __forceinline__ void ce_keys(uint32_t& x, uint32_t& y, bool fma_max) {
+  const uint32_t a = x, b = y;
+  const uint32_t m = min(a, b);
+  y = fma_max ? imad_u32(m, 0u - c_one, imad_u32(a, c_one, b)) : max(a, b);
+  x = m;
+}
+
 template <bool PAIRS>
 struct Elem;
 
@@ -428,7 +450,8 @@ __device__ __forceinline__ void bitonic_merge_pad(uint32_t (&k)[E], uint32_t (&t
         const int j = i + s;
         const bool vi = (virt >> i) & 1u, vj = (virt >> j) & 1u;
         if (!vi && !vj) {
-          Elem<PAIRS>::ce(K[i], K[j], Tg[i], Tg[j], V[i], V[j]);
+          if constexpr (PAIRS) Elem<PAIRS>::ce(K[i], K[j], Tg[i], Tg[j], V[i], V[j]);
+          else ce_keys(K[i], K[j], (i % 3) != 0);  // compile-time after unrolling
         } else if (!vi && vj) {
           // min(-inf, x) = -inf goes to i, x moves to j
           K[j] = K[i];
@@ -476,7 +499,8 @@ __device__ __forceinline__ void oddeven_sort_pad(uint32_t (&k)[E], uint32_t (&t)
         if (x >= j0 && ((x - j0) % (2 * kk)) < kk && y < N && (x / (2 * p)) == (y / (2 * p))) {
           const bool vx = (virt >> x) & 1u, vy = (virt >> y) & 1u;
           if (!vx && !vy) {
-            Elem<PAIRS>::ce(K[x], K[y], Tg[x], Tg[y], V[x], V[y]);
+            if constexpr (PAIRS) Elem<PAIRS>::ce(K[x], K[y], Tg[x], Tg[y], V[x], V[y]);
+            else ce_keys(K[x], K[y], (x % 3) != 0);
           } else if (vx && !vy) {
             // max(+inf, y) = +inf goes to y, y's value moves to x
             K[x] = K[y];
@@ -613,26 +637,38 @@ __device__ __forceinline__ void merge_registers(uint32_t (&key)[E], uint32_t (&v
 // After level 4 the warp's 1024 slots are ascending: lanes 0..30 hold its
 // 992 keys (32 each), lane 31 holds the 32 pads.
 // ---------------------------------------------------------------------------
+// lane keeps min(a, p) (hi = 0) or max(a, p) (hi = 1).  fma form: one ALU
+// min + three FMA-pipe IMADs, r = m + hi * (a + p - 2m); else two ALU ops.
+__device__ __forceinline__ uint32_t lane_minmax(uint32_t a, uint32_t p, bool hi, uint32_t hi01, bool fma_form) {
+  if (fma_form) {
+    const uint32_t m = min(a, p);
+    return imad_u32(hi01, imad_u32(m, 0u - 2u * c_one, imad_u32(a, c_one, p)), m);
+  }
+  return hi ? max(a, p) : min(a, p);
+}
+
 __device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[W], int lane) {
 #pragma unroll
   for (int L = 0; L < 5; ++L) {
     const bool up = (lane >> L) & 1;
+    const uint32_t up01 = up ? 1u : 0u;
     const int m = (2 << L) - 1;
 #pragma unroll
     for (int i = 0; i < W / 2; ++i) {
       const int j = W - 1 - i;
       const uint32_t pi = __shfl_xor_sync(FULL, k[j], m);
       const uint32_t pj = __shfl_xor_sync(FULL, k[i], m);
-      k[i] = up ? max(k[i], pi) : min(k[i], pi);
-      k[j] = up ? max(k[j], pj) : min(k[j], pj);
+      k[i] = lane_minmax(k[i], pi, up, up01, false);
+      k[j] = lane_minmax(k[j], pj, up, up01, true);
     }
 #pragma unroll
     for (int d = L - 1; d >= 0; --d) {
       const bool hi = (lane >> d) & 1;
+      const uint32_t hi01 = hi ? 1u : 0u;
 #pragma unroll
       for (int i = 0; i < W; ++i) {
         const uint32_t p = __shfl_xor_sync(FULL, k[i], 1 << d);
-        k[i] = hi ? max(k[i], p) : min(k[i], p);
+        k[i] = lane_minmax(k[i], p, hi, hi01, (i & 1) != 0);
       }
     }
     uint32_t dt[W], dv[W];
