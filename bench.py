@@ -349,7 +349,16 @@ def main():
                 tr = json.load(f)
             if tr.get("n") == n and tr.get("E") == E and tr.get("u") == u:
                 traffic = tr.get("dram_bytes_per_launch")
+        bs = prof.get("block_sort")
+        in_region = None
+        if bs and bs["launches"] and passes:
+            # the profiled pass brackets every launch with events, which
+            # serialises the launches (no PDL overlap); the headline region has
+            # none: its per-pass time, net of the event-timed block sort
+            in_region = (total_ms_max / a.steps - bs["total_ms"] / bs["launches"]) / passes
         roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "merge_pass_in_region_est_ms": in_region,
+                "achieved_in_region_est": (bytes_per_launch / (in_region / 1e3) / 1e9) if in_region else None,
                 "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
                 "kernel": "merge_pass", "avg_launch_ms": avg_ms, "bytes_per_launch": bytes_per_launch,
                 "peak_source": f"hbm_gbs {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}

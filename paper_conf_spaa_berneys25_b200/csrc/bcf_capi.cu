@@ -129,6 +129,11 @@ static int bs_threads(const Params& p, bool cf, bool pairs) {
     const char* v = getenv("BCF_BS_SAME");
     return v && v[0] == '1';
   }();
+  static const int forced = [] {
+    const char* v = getenv("BCF_BS_THREADS");
+    return v ? atoi(v) : 0;
+  }();
+  if (forced && cf && !pairs && p.E == 31 && u_index(forced) >= 0 && forced >= p.U) return forced;
   if (cf && !pairs && p.E == 31 && p.U == 128 && !same) return 256;
   return p.U;
 }

@@ -162,8 +162,19 @@ __device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uin
 // Block sort (K1): tile t of T = U*E input keys -> sorted run t (descending
 // iff t odd under CF directions).
 // ---------------------------------------------------------------------------
+#ifndef BCF_BS_MINB256
+#define BCF_BS_MINB256 0  // 0: no min-blocks hint (ptxas picks ~80 registers, 3 CTAs/SM)
+#endif
+#ifndef BCF_BS_MINB512
+#define BCF_BS_MINB512 0
+#endif
+template <int U>
+__host__ __device__ constexpr int bs_min_blocks() {
+  return U == 256 ? BCF_BS_MINB256 : (U == 512 ? BCF_BS_MINB512 : 0);
+}
+
 template <int E, int U, bool PAIRS, bool CF>
-__global__ void __launch_bounds__(U) block_sort_kernel(SortArgs args) {
+__global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortArgs args) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
   extern __shared__ __align__(16) uint32_t smem_dyn[];
