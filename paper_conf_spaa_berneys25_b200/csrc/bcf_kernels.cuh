@@ -190,52 +190,69 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortA
   const int cnt = rem < T ? (int)rem : T;
   tma::pdl_wait();  // the input may be produced by the preceding grid
 
-  // --- load: coalesced in physical order, pads = max key (they sort last and
-  // are trimmed by the count; stable order keeps them after real max keys).
-  {
-    const uint32_t* __restrict__ gin_k = args.in_k + t0;
-    const uint32_t* __restrict__ gin_v = PAIRS ? args.in_v + t0 : nullptr;
-    uint32_t vk[E], vv[E];
+  // keys only, E = 31: levels 0..4 (runs up to one warp) run in registers
+  // across the warp (warp_bitonic_levels); any assignment of the warp's 992
+  // keys to its lanes works, so each lane loads its keys straight from global
+  // memory (coalesced: key r of lane l is element 32 r + l of the warp's
+  // chunk) without the shared-memory round trip of the general path
+  constexpr bool WARP_PHASE = CF && !PAIRS && E + 1 == W && U >= 2 * W;
+  uint32_t key[E], val[E], tag[E];
+  if constexpr (WARP_PHASE) {
+    const int wbase = warp * (W * E);
+    const uint32_t* __restrict__ gin_k = args.in_k + t0 + wbase + lane;
+    const int lim = cnt - wbase - lane;  // element 32 r + lane exists iff 32 r < lim
 #pragma unroll
-    for (int r = 0; r < E; ++r) {
-      const int P = tid + r * U;
-      const int p = CF ? rho_inv<E>(P) : P;
-      vk[r] = PAD_KEY;
-      vv[r] = 0;
-      if (p < cnt) {
-        vk[r] = __ldg(gin_k + p);
-        if constexpr (PAIRS) vv[r] = __ldg(gin_v + p);
-      }
-    }
+    for (int r = 0; r < E; ++r) key[r] = (W * r < lim) ? __ldg(gin_k + W * r) : PAD_KEY;
     if (args.encode_f32) {
+#pragma unroll
+      for (int r = 0; r < E; ++r)
+        if (W * r < lim) key[r] = f32_encode(key[r]);
+    }
+  } else {
+    // --- load: coalesced in physical order, pads = max key (they sort last and
+    // are trimmed by the count; stable order keeps them after real max keys).
+    {
+      const uint32_t* __restrict__ gin_k = args.in_k + t0;
+      const uint32_t* __restrict__ gin_v = PAIRS ? args.in_v + t0 : nullptr;
+      uint32_t vk[E], vv[E];
 #pragma unroll
       for (int r = 0; r < E; ++r) {
         const int P = tid + r * U;
         const int p = CF ? rho_inv<E>(P) : P;
-        if (p < cnt) vk[r] = f32_encode(vk[r]);
+        vk[r] = PAD_KEY;
+        vv[r] = 0;
+        if (p < cnt) {
+          vk[r] = __ldg(gin_k + p);
+          if constexpr (PAIRS) vv[r] = __ldg(gin_v + p);
+        }
+      }
+      if (args.encode_f32) {
+#pragma unroll
+        for (int r = 0; r < E; ++r) {
+          const int P = tid + r * U;
+          const int p = CF ? rho_inv<E>(P) : P;
+          if (p < cnt) vk[r] = f32_encode(vk[r]);
+        }
+      }
+#pragma unroll
+      for (int r = 0; r < E; ++r) {
+        sk[tid + r * U] = vk[r];
+        if constexpr (PAIRS) sv[tid + r * U] = vv[r];
       }
     }
+    __syncthreads();
+    // blocked read: round m reads logical tid*E + m (a round set)
 #pragma unroll
-    for (int r = 0; r < E; ++r) {
-      sk[tid + r * U] = vk[r];
-      if constexpr (PAIRS) sv[tid + r * U] = vv[r];
+    for (int m = 0; m < E; ++m) {
+      const int idx = CF ? rho<E>(tid * E + m) : tid * E + m;
+      key[m] = sk[idx];
+      if constexpr (PAIRS) { val[m] = sv[idx]; tag[m] = m; }
     }
-  }
-  __syncthreads();
-  uint32_t key[E], val[E], tag[E];
-  // blocked read: round m reads logical tid*E + m (a round set)
-#pragma unroll
-  for (int m = 0; m < E; ++m) {
-    const int idx = CF ? rho<E>(tid * E + m) : tid * E + m;
-    key[m] = sk[idx];
-    if constexpr (PAIRS) { val[m] = sv[idx]; tag[m] = m; }
   }
   oddeven_sort_pad<E, PAIRS>(key, tag, val);
 
-  // keys only, E = 31: levels 0..4 (runs up to one warp) in registers across
-  // the warp (warp_bitonic_levels), then the warp runs go to shared memory in
-  // the level-5 layout and the CF shared-memory levels continue from l = 5
-  constexpr bool WARP_PHASE = CF && !PAIRS && E + 1 == W && U >= 2 * W;
+  // warp phase, then the warp runs go to shared memory in the level-5 layout
+  // and the CF shared-memory levels continue from l = 5
   int l_first = 0;
   if constexpr (WARP_PHASE) {
     uint32_t k32[W];
@@ -243,7 +260,7 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortA
     for (int i = 0; i < E; ++i) k32[i] = key[i];
     k32[E] = PAD_KEY;
     warp_bitonic_levels(k32, lane);
-    __syncthreads();  // every thread has finished its blocked read of sk
+    __syncthreads();  // (general path: every thread has finished its blocked read of sk)
     warp_run_scatter<E>(sk, k32, warp, lane);
     l_first = 5;
   }

@@ -37,7 +37,10 @@ template <int E, int U>
 __host__ __device__ constexpr int win_stage_words() {
   return ((win_span<E, U>() + E + 8) + 3) / 4 * 4;  // span + cell-scan slack + shift
 }
-constexpr int WIN_STAGES = 2;
+#ifndef BCF_WIN_STAGES
+#define BCF_WIN_STAGES 2
+#endif
+constexpr int WIN_STAGES = BCF_WIN_STAGES;
 template <int E, int U>
 __host__ __device__ constexpr size_t win_smem_bytes() {
   return (size_t)WIN_STAGES * win_stage_words<E, U>() * sizeof(uint32_t);
@@ -77,7 +80,7 @@ __device__ __forceinline__ int warp_prefix_count(int n, P pred, int lane) {
 // resident CTAs per SM the kernel is built for (5 at u = 128)
 template <int U>
 __host__ __device__ constexpr int win_min_blocks() {
-  return U <= 128 ? 5 : (U <= 256 ? 2 : 1);
+  return WIN_STAGES > 2 ? (U <= 128 ? 3 : 1) : (U <= 128 ? 5 : (U <= 256 ? 2 : 1));
 }
 
 template <int E, int U>
@@ -260,13 +263,14 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     if (lane == 0) BCF_TRACE_AT(128 + 2);
     for (int i = 0;; ++i) {
       const int s = i % S;
-      const int s1 = (i + 1) % S;
+      const int s1 = (i + 1) % S;      // stage of the next window
+      const int sp = (i + S - 1) % S;  // stage of subtile i-1 (= s1 for 2 stages)
       if (i >= 1) {
-        // subtile i-1's outputs are staged in s1: stream them out while the
+        // subtile i-1's outputs are staged in sp: stream them out while the
         // consumers search subtile i's split
-        tma::mbar_wait(&empty_bar[s1], (uint32_t)((i - 1) / S) & 1);
+        tma::mbar_wait(&empty_bar[sp], (uint32_t)((i - 1) / S) & 1);
         if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 3);
-        store_out(s1);
+        store_out(sp);
       }
       // subtile i's own end split, found by its consumers
       tma::mbar_wait(&split_bar[s], (uint32_t)(i / S) & 1);
@@ -298,7 +302,12 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
         __syncwarp();
         break;
       }
-      if (lane == 0) tma::bulk_wait_read_all();  // stage s1's store has read it
+      // stage s1's last store (subtile i+1-S) has read it: with 2 stages that
+      // is the store just issued, with more stages an older one
+      if (lane == 0) {
+        if constexpr (S == 2) tma::bulk_wait_read_all();
+        else tma::bulk_wait_read_1();
+      }
       __syncwarp();
       load_window(s1);
       if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 2);
