@@ -144,6 +144,21 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
                               uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes,
                               const bcf_params* p, void* stream);
 
+/* Stable merge of two ascending sorted arrays A = d_a[0, na) and
+   B = d_b[0, nb) into d_out[0, na+nb) (must alias neither); equal keys: all
+   of A's before B's.  The merge step of the pairwise mergesort (merge path,
+   PAPER.md:59-61) as a primitive -- "any parallel scan of a pair of arrays"
+    -- run as ONE pass of the CF merge kernel (conflict-free
+   staging rho(A u pi(B)) and Alg. 1 gather), so no input
+   pair causes a bank conflict.  Values: pass d_a_vals = d_b_vals =
+   d_out_vals = NULL for keys only, else all three (values follow keys).
+   Temp (CUB-style query): 512 bytes (the group descriptor).  na = nb = 0 is
+   a no-op; one side empty is a device copy.  Only BCF_ALGO_CONFLICT_FREE. */
+bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
+                         const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
+                         uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* p,
+                         void* stream);
+
 const char* bcf_status_string(bcf_status s);
 int32_t bcf_abi_version(void);
 /* cudaError_t (as int) of the last BCF_ERROR_CUDA on the calling thread */

@@ -10,6 +10,7 @@ calls raise.
     sort_pairs(keys, values)   stable by u32 key
     worst_case(n, E, u, seed)  Section 4 worst-case permutation (device tensor)
     worst_case_host(...)       same into a numpy array (no CUDA)
+    merge(a, b)                stable merge of two sorted arrays (one CF merge pass)
     split_counts, merge_runs   distributed-sort phases (see dist.py)
 """
 from __future__ import annotations
@@ -34,7 +35,7 @@ ALGO_BASELINE = 1
 EXPORTED_SYMBOLS = [
     "bcf_default_params", "bcf_default_pairs_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
     "bcf_sort_u32_host_batch", "bcf_sort_plan", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
-    "bcf_merge_runs_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
+    "bcf_merge_runs_u32", "bcf_merge_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
     "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
 ]
 
@@ -89,6 +90,8 @@ def lib():
     L.bcf_split_counts_u32.restype = ctypes.c_int
     L.bcf_merge_runs_u32.argtypes = [vp, vp, P(u64), i32, vp, vp, vp, P(sz), P(Params), vp]
     L.bcf_merge_runs_u32.restype = ctypes.c_int
+    L.bcf_merge_u32.argtypes = [vp, u64, vp, u64, vp, vp, vp, vp, vp, P(sz), P(Params), vp]
+    L.bcf_merge_u32.restype = ctypes.c_int
     L.bcf_status_string.argtypes = [ctypes.c_int]
     L.bcf_status_string.restype = ctypes.c_char_p
     L.bcf_abi_version.restype = i32
@@ -306,6 +309,31 @@ def merge_runs(runs, run_offsets, values=None, params: Params | None = None):
                                     out_v.data_ptr() if out_v is not None else None, temp.data_ptr(),
                                     ctypes.byref(tb), pp, _stream(runs)), "bcf_merge_runs_u32")
     return (out, out_v) if values is not None else out
+
+
+def merge(a, b, a_values=None, b_values=None, params: Params | None = None):
+    """Stable merge of two ascending u32 arrays (ties: A first); values follow keys."""
+    torch = _torch()
+    _require_cuda(a, "a")
+    _require_cuda(b, "b")
+    if (a_values is None) != (b_values is None):
+        raise ValueError("pass values for both inputs or for neither")
+    out = torch.empty(a.numel() + b.numel(), dtype=a.dtype, device=a.device)
+    out_v = torch.empty_like(out) if a_values is not None else None
+    L = lib()
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    va = a_values.data_ptr() if a_values is not None else None
+    vb = b_values.data_ptr() if b_values is not None else None
+    vo = out_v.data_ptr() if out_v is not None else None
+    _check(L.bcf_merge_u32(None, a.numel(), None, b.numel(), va, vb, None, vo, None, ctypes.byref(tb), pp, None),
+           "temp query")
+    temp = _temp(tb.value, a.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(a.device):
+        _check(L.bcf_merge_u32(a.data_ptr(), a.numel(), b.data_ptr(), b.numel(), va, vb, out.data_ptr(), vo,
+                               temp.data_ptr(), ctypes.byref(tb), pp, _stream(a)), "bcf_merge_u32")
+    return (out, out_v) if a_values is not None else out
 
 
 def profile_enable(on: bool = True):

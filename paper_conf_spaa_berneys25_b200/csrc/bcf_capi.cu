@@ -529,6 +529,53 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   return BCF_SUCCESS;
 }
 
+bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
+                         const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
+                         uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* pp,
+                         void* stream) {
+  // One CF merge pass (table mode, one group) with B read from its own base
+  // pointer: the merge step of the paper's pairwise mergesort exposed as a
+  // primitive (PAPER.md:59-61 merge path; :380 "any parallel scan of a pair
+  // of arrays").  Ties go to A.
+  if (!temp_bytes) return BCF_ERROR_INVALID_VALUE;
+  const bool pairs = d_a_vals != nullptr || d_b_vals != nullptr || d_out_vals != nullptr;
+  Params p;
+  bcf_status st = resolve(pp, p, pairs);
+  if (st != BCF_SUCCESS) return st;
+  if (p.algo != BCF_ALGO_CONFLICT_FREE) return BCF_ERROR_UNSUPPORTED;
+  const size_t need = 256 + align_up(sizeof(GroupDesc), 256);
+  if (d_temp == nullptr) {
+    *temp_bytes = need;
+    return BCF_SUCCESS;
+  }
+  if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
+  const uint64_t n = na + nb;
+  if (n == 0) return BCF_SUCCESS;
+  if ((na && !d_a) || (nb && !d_b) || !d_out) return BCF_ERROR_INVALID_VALUE;
+  if (pairs && ((na && !d_a_vals) || (nb && !d_b_vals) || !d_out_vals)) return BCF_ERROR_INVALID_VALUE;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (na == 0 || nb == 0) {  // one side empty: the merge is a copy
+    const uint32_t* k = na ? d_a : d_b;
+    const uint32_t* v = na ? d_a_vals : d_b_vals;
+    cudaError_t e = cudaMemcpyAsync(d_out, k, n * 4, cudaMemcpyDeviceToDevice, s);
+    if (e == cudaSuccess && pairs) e = cudaMemcpyAsync(d_out_vals, v, n * 4, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+  }
+  const Variant& var = launch_table().v[p.E][u_index(p.U)][0][pairs ? 1 : 0];
+  if (!var.merge_table) return BCF_ERROR_UNSUPPORTED;
+  const long long T = (long long)p.U * p.E;
+  GroupDesc g{};
+  g.na = (long long)na;
+  g.nb = (long long)nb;
+  GroupDesc* dt = (GroupDesc*)align_up((size_t)d_temp, 256);
+  // pageable source: cudaMemcpyAsync returns once `g` has been staged
+  cudaError_t e = cudaMemcpyAsync(dt, &g, sizeof(g), cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(e);
+  MergeArgs ma{d_a, d_a_vals, d_out, d_out_vals, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, d_b, d_b_vals};
+  e = launch("merge", n, s, [&] { return var.merge_table(ma, (long long)((n + T - 1) / T), s); });
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
 const char* bcf_status_string(bcf_status s) {
   switch (s) {
     case BCF_SUCCESS: return "BCF_SUCCESS";

@@ -66,6 +66,10 @@ struct MergeArgs {
   const GroupDesc* groups;  // table mode (merge of arbitrary runs) if non-null
   int ngroups;
   unsigned long long* trace;  // debug timeline (BCF_TRACE), nullptr normally
+  // table mode, plain kernel only: B runs read from these bases instead of
+  // src_k / src_v (bcf_merge_u32: A and B in separate arrays); nullptr = same
+  const uint32_t* src_kb;
+  const uint32_t* src_vb;
 };
 
 // Group of output tile `tile`: regular pairwise pass (run 2g with run 2g+1,
@@ -391,7 +395,8 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   const GroupDesc grp = group_of_tile(args, tile, T, j);
   const long long lenG = grp.na + grp.nb;
   RunView Av{args.src_k + grp.a_off, grp.na, grp.a_desc};
-  RunView Bv{args.src_k + grp.b_off, grp.nb, grp.b_desc};
+  const uint32_t* __restrict__ baseBk = args.src_kb ? args.src_kb : args.src_k;
+  RunView Bv{baseBk + grp.b_off, grp.nb, grp.b_desc};
   const long long D0 = j * T;
   const long long D1 = D0 + T < lenG ? D0 + T : lenG;
 
@@ -423,9 +428,9 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
     const long long oB = CF ? (BDESC ? grp.b_off + grp.nb - b0 - T : grp.b_off + b0 + T - 1)
                             : grp.b_off + b0 - NA;
     const uint32_t* __restrict__ pAk = args.src_k + oA;
-    const uint32_t* __restrict__ pBk = args.src_k + oB;
+    const uint32_t* __restrict__ pBk = baseBk + oB;
     const uint32_t* __restrict__ pAv = PAIRS ? args.src_v + oA : nullptr;
-    const uint32_t* __restrict__ pBv = PAIRS ? args.src_v + oB : nullptr;
+    const uint32_t* __restrict__ pBv = PAIRS ? (args.src_vb ? args.src_vb : args.src_v) + oB : nullptr;
     const int bstart = CF ? T - NB : NA;
     const int bend = CF ? T : cnt;
     uint32_t vk[E], vv[E];

@@ -103,6 +103,35 @@ def test_temp_query_and_validation():
     assert L.bcf_worst_case_u32_host(out.ctypes.data, 10, 15, 100, 0) == bcf.BCF_ERROR_UNSUPPORTED
 
 
+def test_merge_u32_query_and_validation():
+    L = bcf.lib()
+    tb = ctypes.c_size_t(0)
+    assert L.bcf_merge_u32(None, 100, None, 100, None, None, None, None, None, ctypes.byref(tb), None, None) == 0
+    need = tb.value
+    assert 0 < need <= 1024
+    assert L.bcf_merge_u32(None, 1, None, 1, None, None, None, None, None, None, None,
+                           None) == bcf.BCF_ERROR_INVALID_VALUE
+    small = ctypes.c_size_t(need - 1)
+    assert L.bcf_merge_u32(None, 1, None, 1, None, None, None, None, ctypes.c_void_p(256), ctypes.byref(small),
+                           None, None) == bcf.BCF_ERROR_TEMP_TOO_SMALL
+    tb = ctypes.c_size_t(need)
+    tmp = ctypes.c_void_p(256)
+    # na = nb = 0 is a no-op; null inputs / output with data are rejected before any launch
+    assert L.bcf_merge_u32(None, 0, None, 0, None, None, None, None, tmp, ctypes.byref(tb), None, None) == 0
+    fake = ctypes.c_void_p(4096)
+    assert L.bcf_merge_u32(None, 5, fake, 5, None, None, fake, None, tmp, ctypes.byref(tb), None,
+                           None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_merge_u32(fake, 5, fake, 5, None, None, None, None, tmp, ctypes.byref(tb), None,
+                           None) == bcf.BCF_ERROR_INVALID_VALUE
+    # values: all three or none
+    assert L.bcf_merge_u32(fake, 5, fake, 5, fake, None, fake, fake, tmp, ctypes.byref(tb), None,
+                           None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_merge_u32(None, 5, None, 5, None, None, None, None, None, ctypes.byref(tb),
+                           bcf.make_params(15, 256, bcf.ALGO_BASELINE), None) == bcf.BCF_ERROR_UNSUPPORTED
+    assert L.bcf_merge_u32(None, 5, None, 5, None, None, None, None, None, ctypes.byref(tb),
+                           bcf.make_params(18, 256), None) == bcf.BCF_ERROR_UNSUPPORTED
+
+
 @pytest.mark.parametrize("E,u,n,seed", [
     (15, 64, 15 * 2 ** 9, 1234), (17, 64, 17 * 2 ** 9, 5), (16, 64, 2 ** 13, 7), (12, 64, 12 * 2 ** 9, 9),
     (8, 128, 2 ** 13, 11), (15, 256, 100000, 3), (16, 256, 2 ** 16, 0xB2000000), (9, 128, 7777, 1),

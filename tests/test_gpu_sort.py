@@ -208,6 +208,48 @@ def test_merge_runs_stable(sizes):
     np.testing.assert_array_equal(to_host(k_only), ek)
 
 
+MERGE_SIZES = [(0, 0), (0, 5), (7, 0), (1, 1), (3968 * 3 + 17, 5000), (100000, 1), (1, 100000),
+               (70001, 70003), (4352, 4352), (1 << 20, (1 << 20) - 3)]
+
+
+@pytest.mark.parametrize("na,nb", MERGE_SIZES)
+@pytest.mark.parametrize("dist", ["dups", "uniform", "disjoint"])
+def test_merge_two_arrays(na, nb, dist):
+    """bcf_merge_u32 == stable sort of A ++ B (ties: A first), keys and pairs,
+    default and pairs parameters; A and B in separate allocations."""
+    rng = np.random.default_rng(na * 7 + nb + len(dist))
+    if dist == "dups":
+        a = rng.integers(0, 50, size=na).astype(np.uint32)
+        b = rng.integers(0, 50, size=nb).astype(np.uint32)
+    elif dist == "uniform":
+        a = si.uniform_u32(na, si.config_seed(0))
+        b = si.uniform_u32(nb, si.config_seed(0), lo=na)
+    else:  # every B key below every A key: the merge path runs along one edge
+        a = rng.integers(1 << 31, 1 << 32, size=na, dtype=np.uint64).astype(np.uint32)
+        b = rng.integers(0, 1 << 31, size=nb, dtype=np.uint64).astype(np.uint32)
+    a.sort(kind="stable")
+    b.sort(kind="stable")
+    cat = np.concatenate([a, b])
+    idx = np.arange(na + nb, dtype=np.uint32)
+    ek, ev = oracle.sort_pairs_u32(cat, idx)
+    ko = bcf.merge(to_dev(a), to_dev(b))
+    np.testing.assert_array_equal(to_host(ko), ek)
+    for params in (None, bcf.make_params(15, 256)):
+        ko, vo = bcf.merge(to_dev(a), to_dev(b), to_dev(idx[:na]), to_dev(idx[na:]), params=params)
+        np.testing.assert_array_equal(to_host(ko), ek)
+        np.testing.assert_array_equal(to_host(vo), ev)
+
+
+def test_merge_unaligned_views():
+    rng = np.random.default_rng(3)
+    a = np.sort(rng.integers(0, 1000, size=20001).astype(np.uint32))
+    b = np.sort(rng.integers(0, 1000, size=30003).astype(np.uint32))
+    da = to_dev(np.concatenate([[7], a]))[1:]
+    db = to_dev(np.concatenate([[1, 2, 3], b]))[3:]
+    ek, _ = oracle.sort_pairs_u32(np.concatenate([a, b]), np.arange(a.size + b.size, dtype=np.uint32))
+    np.testing.assert_array_equal(to_host(bcf.merge(da, db)), ek)
+
+
 # ---- full BASELINE sizes, bench launch configuration ------------------------
 
 def test_full_2p24_random_and_worst():
