@@ -152,6 +152,8 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
    staging rho(A u pi(B)) and Alg. 1 gather), so no input
    pair causes a bank conflict.  Values: pass d_a_vals = d_b_vals =
    d_out_vals = NULL for keys only, else all three (values follow keys).
+   Precondition: A and B ascending (not checked -- that would cost a pass;
+   unsorted inputs are undefined behaviour, as for any merge-path merge).
    Temp (CUB-style query): 512 bytes (the group descriptor).  na = nb = 0 is
    a no-op; one side empty is a device copy.  Only BCF_ALGO_CONFLICT_FREE. */
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,

@@ -244,8 +244,9 @@ def test_merge_unaligned_views():
     rng = np.random.default_rng(3)
     a = np.sort(rng.integers(0, 1000, size=20001).astype(np.uint32))
     b = np.sort(rng.integers(0, 1000, size=30003).astype(np.uint32))
-    da = to_dev(np.concatenate([[7], a]))[1:]
-    db = to_dev(np.concatenate([[1, 2, 3], b]))[3:]
+    da = to_dev(np.concatenate([np.array([7], np.uint32), a]))[1:]
+    db = to_dev(np.concatenate([np.array([1, 2, 3], np.uint32), b]))[3:]
+    assert da.numel() == a.size and db.numel() == b.size
     ek, _ = oracle.sort_pairs_u32(np.concatenate([a, b]), np.arange(a.size + b.size, dtype=np.uint32))
     np.testing.assert_array_equal(to_host(bcf.merge(da, db)), ek)
 

@@ -13,7 +13,7 @@
 // Build: nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a
 //        tools/cub_contrast.cu -Iinclude -Lpaper_conf_spaa_berneys25_b200 -lbcf
 //        -Xlinker -rpath -Xlinker $PWD/paper_conf_spaa_berneys25_b200 -o tools/cub_contrast
-// Run:   tools/cub_contrast [log2n=24] [reps=20]   -> one JSON line on stdout
+// Run:   tools/cub_contrast [log2n=24 | n] [reps=20]   -> one JSON line on stdout
 #include <cub/device/device_merge_sort.cuh>
 #include <cub/device/device_radix_sort.cuh>
 #include <cuda_runtime.h>
@@ -60,9 +60,9 @@ static double median(std::vector<double> v) {
 }
 
 int main(int argc, char** argv) {
-  const int lg = argc > 1 ? atoi(argv[1]) : 24;
+  const long long arg = argc > 1 ? atoll(argv[1]) : 24;  // log2(n) if <= 40, else n
   const int reps = argc > 2 ? atoi(argv[2]) : 20;
-  const uint64_t n = 1ull << lg;
+  const uint64_t n = arg <= 40 ? 1ull << arg : (uint64_t)arg;
   const uint64_t seed = 0xB2000000ull + 1;  // BASELINE configs[1]
   std::vector<uint32_t> h_rand(n), h_worst(n), h_a(n), h_b(n);
   for (uint64_t i = 0; i < n; ++i) h_rand[i] = (uint32_t)(mix64(seed + (i + 1) * 0x9E3779B97F4A7C15ull) >> 32);
