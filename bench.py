@@ -153,6 +153,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
     legs = [
         ("f32_2^28", 1 << 28, 8),
         ("pairs_u32_2^26", 1 << 26, 16),
+        ("merge_u32_2x2^25", 1 << 26, 8),
     ]
     for name, n, bpk in legs:
         if name.startswith("f32"):
@@ -160,6 +161,15 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             out = torch.empty_like(x)
             run = lambda: bcf.sort(x, out=out, params=params, temp=temp)  # noqa: E731
             workload = "2^28 float32 keys, uniform [0,1) (24-bit mantissa grid), IEEE totalOrder"
+        elif name.startswith("merge"):
+            # bcf_merge_u32: two separately allocated sorted halves
+            prm = params
+            ka = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(5), dev), params=prm)
+            kb = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(5), dev, lo=n // 2), params=prm)
+            mo = torch.empty(n, dtype=ka.dtype, device=dev)
+            mtemp = bcf._temp(1024, dev)
+            run = lambda: bcf.merge(ka, kb, params=prm, out=mo, temp=mtemp)  # noqa: E731
+            workload = "bcf_merge_u32 of two sorted 2^25 uniform uint32 arrays (one CF merge pass, table mode)"
         else:
             k = si.dup_u32_torch(n, si.config_seed(4), dev)
             v = si.iota_u32_torch(n, dev)
@@ -167,7 +177,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             prm = bcf.default_pairs_params()  # pairs default (17, 256)
             run = lambda: bcf.sort_pairs(k, v, ko, vo, params=prm, temp=temp)  # noqa: E731
             workload = "2^26 uint32 (key & 0xFFFF, heavy duplicates) + uint32 value (index) pairs, stable"
-        if name.startswith("f32"):
+        if name.startswith("f32") or name.startswith("merge"):
             prm = params
         temp = bcf.temp_buffer(n, prm, pairs=name.startswith("pairs"), device=dev)
         for _ in range(3):
@@ -188,7 +198,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         torch.cuda.synchronize()
         bcf.profile_enable(False)
         prof = bcf.profile_collect()
-        mp = prof.get("merge_pass", {"launches": 0, "total_ms": 0.0})
+        mp = prof.get("merge" if name.startswith("merge") else "merge_pass", {"launches": 0, "total_ms": 0.0})
         bs = prof.get("block_sort", {"launches": 0, "total_ms": 0.0})
         avg = mp["total_ms"] / max(1, mp["launches"])
         res[name] = {"workload": workload, "n": n, "E": prm.items_per_thread, "u": prm.block_threads,

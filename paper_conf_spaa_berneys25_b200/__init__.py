@@ -311,29 +311,36 @@ def merge_runs(runs, run_offsets, values=None, params: Params | None = None):
     return (out, out_v) if values is not None else out
 
 
-def merge(a, b, a_values=None, b_values=None, params: Params | None = None):
+def merge(a, b, a_values=None, b_values=None, params: Params | None = None, out=None, out_values=None,
+          temp=None):
     """Stable merge of two ascending u32 arrays (ties: A first); values follow keys."""
     torch = _torch()
     _require_cuda(a, "a")
     _require_cuda(b, "b")
     if (a_values is None) != (b_values is None):
         raise ValueError("pass values for both inputs or for neither")
-    out = torch.empty(a.numel() + b.numel(), dtype=a.dtype, device=a.device)
-    out_v = torch.empty_like(out) if a_values is not None else None
+    if out is None:
+        out = torch.empty(a.numel() + b.numel(), dtype=a.dtype, device=a.device)
+    _require_cuda(out, "out")
+    if out.numel() != a.numel() + b.numel():
+        raise ValueError("out must hold a.numel() + b.numel() keys")
+    if a_values is not None and out_values is None:
+        out_values = torch.empty_like(out)
     L = lib()
     tb = ctypes.c_size_t(0)
     pp = ctypes.byref(params) if params is not None else None
     va = a_values.data_ptr() if a_values is not None else None
     vb = b_values.data_ptr() if b_values is not None else None
-    vo = out_v.data_ptr() if out_v is not None else None
+    vo = out_values.data_ptr() if a_values is not None else None
     _check(L.bcf_merge_u32(None, a.numel(), None, b.numel(), va, vb, None, vo, None, ctypes.byref(tb), pp, None),
            "temp query")
-    temp = _temp(tb.value, a.device)
+    if temp is None or temp.numel() < tb.value:
+        temp = _temp(tb.value, a.device)
     tb = ctypes.c_size_t(temp.numel())
     with torch.cuda.device(a.device):
         _check(L.bcf_merge_u32(a.data_ptr(), a.numel(), b.data_ptr(), b.numel(), va, vb, out.data_ptr(), vo,
                                temp.data_ptr(), ctypes.byref(tb), pp, _stream(a)), "bcf_merge_u32")
-    return (out, out_v) if a_values is not None else out
+    return (out, out_values) if a_values is not None else out
 
 
 def profile_enable(on: bool = True):
