@@ -294,12 +294,16 @@ def main():
     temp = torch.empty(tb.value, dtype=torch.uint8, device=dev)
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
 
-    def step(i):
+    dist_marks, dist_sends = [], []
+
+    def step(i, timing=None):
         x = inputs[i % 2]
         if world == 1:
             bcf.sort(x, out=out, params=params, temp=temp)
         else:
-            bdist.sort(x, ops=bdist.CudaOps(params))
+            _, _, st = bdist.sort(x, ops=bdist.CudaOps(params), timing=timing)
+            if timing is not None:
+                dist_sends.append(st.send_counts)
 
     for i in range(max(3, a.warmup)):
         step(i)
@@ -327,10 +331,32 @@ def main():
     bcf.profile_enable(True)
     for i in range(min(a.steps, 50)):
         flush.fill_(i)
-        step(i)
+        step(i, timing=dist_marks if world > 1 else None)
     torch.cuda.synchronize()
     bcf.profile_enable(False)
     prof = bcf.profile_collect()
+    distributed = None
+    if world > 1 and dist_marks:
+        # phase split of the distributed sort, from CUDA events
+        # on the launch stream in the profiled pass; max over ranks.  Exchange
+        # bandwidth = this rank's off-rank key bytes out / exchange time, against
+        # NVLink 5's 900 GB/s per direction per GPU.
+        names = list(bdist._PhaseMarks.NAMES)
+        ph = [m.phase_ms() for m in dist_marks]
+        mean_ms = [statistics.mean(p_[k] for p_ in ph) for k in names]
+        offrank = statistics.mean(4 * (sum(sc) - sc[rank]) for sc in dist_sends)
+        ex_rate = offrank / (mean_ms[names.index("exchange")] / 1e3) / 1e9
+        tt = torch.tensor(mean_ms + [-ex_rate], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ph_max = tt.tolist()
+        slowest = -ph_max[-1]  # min over ranks of the exchange rate
+        distributed = {
+            "phases_ms_max_over_ranks": dict(zip(names, ph_max[:-1])),
+            "exchange": {"achieved_gbs_min_over_ranks": slowest, "peak": 900.0, "unit": "GB/s",
+                         "frac": slowest / 900.0, "offrank_bytes_out_rank0": offrank,
+                         "peak_source": "NVLink 5 per direction per GPU (nominal)"},
+            "splitters": "exact, 64-ary bisection of the key space + rank-ordered tie split",
+        }
     prof_ms = sum(v["total_ms"] for v in prof.values())
     ms = [s.elapsed_time(e) for s, e in ev]
     total_ms = sum(ms)
@@ -393,6 +419,8 @@ def main():
         "gpu_launches": launches,
         "clocks": clk.summary(),
     }
+    if distributed is not None:
+        line["distributed"] = distributed
 
     if rank == 0 and world == 1 and not a.no_extras:
         # e2e through the public C-ABI host-buffer entry point

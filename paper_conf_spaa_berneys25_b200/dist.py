@@ -129,30 +129,66 @@ def exact_splitters(sorted_keys, n_local: int, group, ops, device):
     return send, [int(v) for v in vs], rounds
 
 
-def sort(keys, values=None, group=None, ops=None):
+class _PhaseMarks:
+    """CUDA events on the current stream at the phase boundaries of one
+    distributed sort (local_sort | splitters | exchange | merge); a no-op for
+    non-CUDA tensors (gloo tests).  Read with phase_ms() after a synchronize."""
+
+    NAMES = ("local_sort", "splitters", "exchange", "merge")
+
+    def __init__(self, device, enabled: bool):
+        import torch
+
+        self.on = enabled and device.type == "cuda"
+        self.ev = []
+        self._torch = torch
+        self.device = device
+
+    def mark(self):
+        if self.on:
+            e = self._torch.cuda.Event(enable_timing=True)
+            e.record(self._torch.cuda.current_stream(self.device))
+            self.ev.append(e)
+
+    def phase_ms(self) -> dict:
+        if len(self.ev) != len(self.NAMES) + 1:
+            return {}
+        return {n: self.ev[i].elapsed_time(self.ev[i + 1]) for i, n in enumerate(self.NAMES)}
+
+
+def sort(keys, values=None, group=None, ops=None, timing: list | None = None):
     """Distributed stable sort of the shards held by the ranks of `group`.
     Returns (keys_out, values_out_or_None, DistStats).  keys: 1-D 4-byte
-    tensor (u32 bit patterns in int32); values likewise."""
+    tensor (u32 bit patterns in int32); values likewise.  `timing`: if a
+    list, a _PhaseMarks of this call is appended (CUDA tensors only)."""
     import torch
     import torch.distributed as dist
 
     ops = ops or CudaOps()
     device = keys.device
     p = dist.get_world_size(group)
+    marks = _PhaseMarks(device, timing is not None and p > 1)
+    marks.mark()
     sk, sv = ops.sort(keys, values)
     if p == 1:
         return sk, sv, DistStats(0, [keys.numel()], [keys.numel()], [])
+    marks.mark()
     send, pivots, rounds = exact_splitters(sk, sk.numel(), group, ops, device)
     sc = torch.tensor(send, dtype=torch.int64, device=device)
     rc = torch.empty_like(sc)
     dist.all_to_all_single(rc, sc, group=group)
     recv = [int(x) for x in rc.cpu().tolist()]
+    marks.mark()
     rk = torch.empty(sum(recv), dtype=keys.dtype, device=device)
     dist.all_to_all_single(rk, sk, output_split_sizes=recv, input_split_sizes=send, group=group)
     rv = None
     if sv is not None:
         rv = torch.empty(sum(recv), dtype=values.dtype, device=device)
         dist.all_to_all_single(rv, sv, output_split_sizes=recv, input_split_sizes=send, group=group)
+    marks.mark()
     offs = np.concatenate([[0], np.cumsum(recv)]).astype(np.uint64)
     ok, ov = ops.merge_runs(rk, offs, rv)
+    marks.mark()
+    if timing is not None:
+        timing.append(marks)
     return ok, ov, DistStats(rounds, send, recv, pivots)

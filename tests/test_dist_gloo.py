@@ -61,7 +61,9 @@ def _worker(rank, world, port, case, q):
         vals = si.iota_u32(hi - lo, lo=lo)
         kt = torch.from_numpy(keys.view(np.int32).copy())
         vt = torch.from_numpy(vals.view(np.int32).copy()) if with_vals else None
-        ok, ov, st = bdist.sort(kt, vt, ops=NumpyOps())
+        tm = []
+        ok, ov, st = bdist.sort(kt, vt, ops=NumpyOps(), timing=tm)
+        assert len(tm) == 1 and tm[0].phase_ms() == {}  # phase events are CUDA-only
         q.put((rank, ok.numpy().view(np.uint32).copy(),
                None if ov is None else ov.numpy().view(np.uint32).copy(), st.rounds))
     finally:
