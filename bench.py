@@ -167,9 +167,10 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             ka = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(5), dev), params=prm)
             kb = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(5), dev, lo=n // 2), params=prm)
             mo = torch.empty(n, dtype=ka.dtype, device=dev)
-            mtemp = bcf._temp(1024, dev)
+            mtemp = bcf.merge_temp(n // 2, n // 2, params=prm, device=dev)
             run = lambda: bcf.merge(ka, kb, params=prm, out=mo, temp=mtemp)  # noqa: E731
-            workload = "bcf_merge_u32 of two sorted 2^25 uniform uint32 arrays (one CF merge pass, table mode)"
+            workload = ("bcf_merge_u32 of two sorted 2^25 uniform uint32 arrays (B reversed into temp, then one "
+                        "pass of the window merge kernel)")
         else:
             k = si.dup_u32_torch(n, si.config_seed(4), dev)
             v = si.iota_u32_torch(n, dev)

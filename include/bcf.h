@@ -154,8 +154,14 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
    d_out_vals = NULL for keys only, else all three (values follow keys).
    Precondition: A and B ascending (not checked -- that would cost a pass;
    unsorted inputs are undefined behaviour, as for any merge-path merge).
-   Temp (CUB-style query): 512 bytes (the group descriptor).  na = nb = 0 is
-   a no-op; one side empty is a device copy.  Only BCF_ALGO_CONFLICT_FREE. */
+   Keys only, E coprime with 32 and d_a 16-byte aligned: B is first reversed
+   into temp (the persistent window kernel bulk-copies B windows into their
+   reversed slots, so it needs B stored descending: +8 B of traffic per B
+   key), then one pass of the window kernel; otherwise one pass of the plain
+   LSU-staged CF kernel reading B ascending.  Temp (CUB-style query): 512
+   bytes (group descriptor), + 4 (nb + 8) bytes (rounded up to 256) for keys
+   only.  na = nb = 0 is a no-op; one side empty is a device copy.  Only
+   BCF_ALGO_CONFLICT_FREE. */
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
                          const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
                          uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* p,

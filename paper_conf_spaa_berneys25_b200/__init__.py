@@ -311,6 +311,16 @@ def merge_runs(runs, run_offsets, values=None, params: Params | None = None):
     return (out, out_v) if values is not None else out
 
 
+def merge_temp(na: int, nb: int, pairs: bool = False, params: Params | None = None, device="cuda"):
+    """Temp storage for bcf_merge_u32 of na + nb keys (or pairs)."""
+    tb = ctypes.c_size_t(0)
+    pp = ctypes.byref(params) if params is not None else None
+    vo = ctypes.c_void_p(16) if pairs else None  # only the pairs flag matters for the query
+    _check(lib().bcf_merge_u32(None, na, None, nb, vo, vo, None, vo, None, ctypes.byref(tb), pp, None),
+           "temp query")
+    return _temp(tb.value, device)
+
+
 def merge(a, b, a_values=None, b_values=None, params: Params | None = None, out=None, out_values=None,
           temp=None):
     """Stable merge of two ascending u32 arrays (ties: A first); values follow keys."""

@@ -529,6 +529,13 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   return BCF_SUCCESS;
 }
 
+// B reversed into temp for the window kernel, whose bulk copies need B
+// stored descending (element y of B at out[nb-1-y])
+__global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, long long n) {
+  for (long long j = blockIdx.x * (long long)blockDim.x + threadIdx.x; j < n; j += (long long)gridDim.x * blockDim.x)
+    out[j] = __ldg(in + (n - 1 - j));
+}
+
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
                          const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
                          uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* pp,
@@ -543,7 +550,8 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
   bcf_status st = resolve(pp, p, pairs);
   if (st != BCF_SUCCESS) return st;
   if (p.algo != BCF_ALGO_CONFLICT_FREE) return BCF_ERROR_UNSUPPORTED;
-  const size_t need = 256 + align_up(sizeof(GroupDesc), 256);
+  // keys only: room for B reversed (window kernel path), +8 words of phase/tail slack
+  const size_t need = 256 + align_up(sizeof(GroupDesc), 256) + (pairs ? 0 : align_up(4 * ((size_t)nb + 8), 256));
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -564,15 +572,35 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
   const Variant& var = launch_table().v[p.E][u_index(p.U)][0][pairs ? 1 : 0];
   if (!var.merge_table) return BCF_ERROR_UNSUPPORTED;
   const long long T = (long long)p.U * p.E;
+  const long long tiles = (long long)((n + T - 1) / T);
   GroupDesc g{};
   g.na = (long long)na;
   g.nb = (long long)nb;
   GroupDesc* dt = (GroupDesc*)align_up((size_t)d_temp, 256);
+  if (!pairs && var.merge_win && ((uintptr_t)d_a & 15) == 0 && !tma_disabled()) {
+    // persistent window kernel (0.8 of HBM per pass at 2^28): B reversed into
+    // temp at word phase b_off = -nb mod 4, so that A's and B's windows share
+    // one 16-byte phase (a_off - b_off - nb = 0 mod 4, as in the sort's passes)
+    uint32_t* rb = (uint32_t*)((char*)dt + align_up(sizeof(GroupDesc), 256));
+    g.b_off = (long long)((4 - (nb & 3)) & 3);
+    g.b_desc = 1;
+    cudaError_t e = cudaMemcpyAsync(dt, &g, sizeof(g), cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(e);
+    const long long blocks = std::min<long long>((long long)((nb + 255) / 256), 148LL * 16);
+    e = launch("merge_reverse", nb, s, [&] {
+      reverse_u32_kernel<<<(unsigned)blocks, 256, 0, s>>>(d_b, rb + g.b_off, (long long)nb);
+      return cudaGetLastError();
+    });
+    if (e != cudaSuccess) return cuda_fail(e);
+    MergeArgs ma{d_a, nullptr, d_out, nullptr, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, rb, nullptr};
+    e = launch("merge", n, s, [&] { return var.merge_win(ma, tiles, s); });
+    return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+  }
   // pageable source: cudaMemcpyAsync returns once `g` has been staged
   cudaError_t e = cudaMemcpyAsync(dt, &g, sizeof(g), cudaMemcpyHostToDevice, s);
   if (e != cudaSuccess) return cuda_fail(e);
   MergeArgs ma{d_a, d_a_vals, d_out, d_out_vals, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, d_b, d_b_vals};
-  e = launch("merge", n, s, [&] { return var.merge_table(ma, (long long)((n + T - 1) / T), s); });
+  e = launch("merge", n, s, [&] { return var.merge_table(ma, tiles, s); });
   return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
 }
 

@@ -122,6 +122,8 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
   if (warp == NW) {
     // =========================== producer ===========================
     const uint32_t* __restrict__ src = args.src_k;
+    // B runs (table mode, bcf_merge_u32): a separate base, stored descending
+    const uint32_t* __restrict__ srcB = args.src_kb ? args.src_kb : args.src_k;
     const long long dst_phase = (long long)(((uintptr_t)args.dst_k >> 2) & 3);
 
     // current segment: the part of one merge group inside this CTA's range
@@ -139,7 +141,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     long long a0;
     {
       RunView Av{src + grp.a_off, grp.na, 0};
-      RunView Bv{src + grp.b_off, grp.nb, 1};
+      RunView Bv{srcB + grp.b_off, grp.nb, 1};
       const long long lenG = grp.na + grp.nb;
       const long long guess = lenG > 0 ? (long long)((double)D0 * (double)grp.na / (double)lenG) : 0;
       a0 = j0 == 0 ? 0 : merge_path_warp_global_guess(Av, Bv, D0, 0, D0, guess, lane);
@@ -199,6 +201,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       // edge words first (their loads overlap the bulk-copy issue)
       int w = -1;
       long long gw = 0;
+      const uint32_t* __restrict__ esrc = lane >= 4 ? srcB : src;
       if (lane >= 1 && lane <= 3 && ea0 + lane - 1 < ea1) {
         w = ea0 + lane - 1;
         gw = oA + (w - c);
@@ -209,7 +212,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       if (lane == 0) {
         tma::mbar_expect_tx(&full_bar[s], (uint32_t)(a_hi + (b_hi - b_lo)) * 4u);
         if (a_hi > 0) tma::bulk_g2s(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
-        if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, src + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, srcB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
         // L2 prefetch of the keys the next window will need beyond this one
         // (both runs are consumed sequentially): the next window's bulk loads,
         // issued one subtile later, then hit L2 instead of DRAM
@@ -223,9 +226,9 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
         long long pb0 = grp.b_off;
         if (pb0 < pb1 - PF) pb0 = pb1 - PF;
         pb0 = (pb0 + 3) & ~3ll;
-        if (pb1 > pb0) tma::bulk_prefetch_l2(src + pb0, (uint32_t)(pb1 - pb0) * 4u);
+        if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
       }
-      const uint32_t ev = w >= 0 ? __ldg(src + gw) : 0u;
+      const uint32_t ev = w >= 0 ? __ldg(esrc + gw) : 0u;
       if (w >= 0) sk[w] = ev;
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);

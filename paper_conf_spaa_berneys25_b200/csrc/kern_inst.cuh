@@ -124,6 +124,14 @@ cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s
   }
 }
 
+// the window kernel alone (keys only; bcf_merge_u32 passes B through src_kb,
+// which only the window and plain kernels read)
+template <int E, int U>
+cudaError_t launch_merge_win(const MergeArgs& a, long long tiles, cudaStream_t s) {
+  static PersistentCache pc;
+  return launch_persistent(merge_pass_win_kernel<E, U>, pc, win_smem_bytes<E, U>(), U + 32, a, tiles, s);
+}
+
 template <int E, int U>
 void register_eu(LaunchTable& t) {
   const int ui = u_index(U);
@@ -136,6 +144,8 @@ void register_eu(LaunchTable& t) {
   if constexpr (cgcd(W, E) == 1) {
     t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
     t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
+      t.v[E][ui][0][0].merge_win = &launch_merge_win<E, U>;
   }
 }
 

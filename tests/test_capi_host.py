@@ -108,11 +108,15 @@ def test_merge_u32_query_and_validation():
     tb = ctypes.c_size_t(0)
     assert L.bcf_merge_u32(None, 100, None, 100, None, None, None, None, None, ctypes.byref(tb), None, None) == 0
     need = tb.value
-    assert 0 < need <= 1024
+    assert 0 < need <= 1024 + 4 * 100
+    tbp = ctypes.c_size_t(0)
+    fake0 = ctypes.c_void_p(4096)
+    assert L.bcf_merge_u32(None, 100, None, 100, fake0, fake0, None, fake0, None, ctypes.byref(tbp), None,
+                           None) == 0 and 0 < tbp.value <= 1024
     assert L.bcf_merge_u32(None, 1, None, 1, None, None, None, None, None, None, None,
                            None) == bcf.BCF_ERROR_INVALID_VALUE
     small = ctypes.c_size_t(need - 1)
-    assert L.bcf_merge_u32(None, 1, None, 1, None, None, None, None, ctypes.c_void_p(256), ctypes.byref(small),
+    assert L.bcf_merge_u32(None, 100, None, 100, None, None, None, None, ctypes.c_void_p(256), ctypes.byref(small),
                            None, None) == bcf.BCF_ERROR_TEMP_TOO_SMALL
     tb = ctypes.c_size_t(need)
     tmp = ctypes.c_void_p(256)

@@ -232,8 +232,11 @@ def test_merge_two_arrays(na, nb, dist):
     cat = np.concatenate([a, b])
     idx = np.arange(na + nb, dtype=np.uint32)
     ek, ev = oracle.sort_pairs_u32(cat, idx)
-    ko = bcf.merge(to_dev(a), to_dev(b))
-    np.testing.assert_array_equal(to_host(ko), ek)
+    # keys only: window kernel (odd E, aligned A; B reversed into temp) and
+    # the plain kernel (even E: rho != identity)
+    for params in (None, bcf.make_params(15, 256), bcf.make_params(16, 128), bcf.make_params(31, 512)):
+        ko = bcf.merge(to_dev(a), to_dev(b), params=params)
+        np.testing.assert_array_equal(to_host(ko), ek)
     for params in (None, bcf.make_params(15, 256)):
         ko, vo = bcf.merge(to_dev(a), to_dev(b), to_dev(idx[:na]), to_dev(idx[na:]), params=params)
         np.testing.assert_array_equal(to_host(ko), ek)
