@@ -154,6 +154,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         ("f32_2^28", 1 << 28, 8),
         ("pairs_u32_2^26", 1 << 26, 16),
         ("merge_u32_2x2^25", 1 << 26, 8),
+        ("merge_runs_8x2^23", 1 << 26, 24),  # 3 pairwise passes x 8 B/key
     ]
     for name, n, bpk in legs:
         if name.startswith("f32"):
@@ -161,6 +162,14 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             out = torch.empty_like(x)
             run = lambda: bcf.sort(x, out=out, params=params, temp=temp)  # noqa: E731
             workload = "2^28 float32 keys, uniform [0,1) (24-bit mantissa grid), IEEE totalOrder"
+        elif name.startswith("merge_runs"):
+            # bcf_merge_runs_u32: the distributed sort's final local merge at p = 8
+            prm = params
+            rk = torch.cat([bcf.sort(si.uniform_u32_torch(n // 8, si.config_seed(6), dev, lo=r * (n // 8)),
+                                     params=prm) for r in range(8)])
+            roffs = np.arange(9, dtype=np.uint64) * np.uint64(n // 8)
+            run = lambda: bcf.merge_runs(rk, roffs, params=prm)  # noqa: E731
+            workload = "bcf_merge_runs_u32 of 8 sorted 2^23 uniform uint32 runs (3 CF merge passes)"
         elif name.startswith("merge"):
             # bcf_merge_u32: two separately allocated sorted halves
             prm = params
@@ -199,16 +208,23 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         torch.cuda.synchronize()
         bcf.profile_enable(False)
         prof = bcf.profile_collect()
-        mp = prof.get("merge" if name.startswith("merge") else "merge_pass", {"launches": 0, "total_ms": 0.0})
+        cls = "merge_runs" if name.startswith("merge_runs") else ("merge" if name.startswith("merge") else "merge_pass")
+        mp = prof.get(cls, {"launches": 0, "total_ms": 0.0})
         bs = prof.get("block_sort", {"launches": 0, "total_ms": 0.0})
         avg = mp["total_ms"] / max(1, mp["launches"])
         res[name] = {"workload": workload, "n": n, "E": prm.items_per_thread, "u": prm.block_threads,
                      "value": n / (ms / 1e3),
                      "unit": "pairs/s" if name.startswith("pairs") else "keys/s", "ms_per_sort": ms,
                      "merge_pass": {"launches_per_sort": mp["launches"] // 3, "avg_ms": avg,
+                                    "achieved_gbs": 8 * n / (avg / 1e3) / 1e9 if avg else None,
+                                    "frac_of_hbm": (8 * n / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
+                                    "bytes_per_launch": 8 * n} if name.startswith("merge_runs") else
+                                   {"launches_per_sort": mp["launches"] // 3, "avg_ms": avg,
                                     "achieved_gbs": bpk * n / (avg / 1e3) / 1e9 if avg else None,
                                     "frac_of_hbm": (bpk * n / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
                                     "bytes_per_launch": bpk * n},
+                     # merge legs: algorithmic bytes of the whole call / call time
+                     "call_gbs_algorithmic": bpk * n / (ms / 1e3) / 1e9 if name.startswith("merge") else None,
                      "block_sort_ms": bs["total_ms"] / max(1, bs["launches"])}
         del run, temp
         torch.cuda.empty_cache()

@@ -458,7 +458,13 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
                               int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals, void* d_temp,
                               size_t* temp_bytes, const bcf_params* pp, void* stream) {
   // Pairwise merge tree over the runs in run order (run 2g is A, 2g+1 is B,
-  // ties to A = the lower run), table mode of the CF merge-pass kernel.
+  // ties to A = the lower run).  Pass 1 reads the caller's ascending runs with
+  // the plain table-mode kernel; it and every later non-final pass write odd
+  // groups DESCENDING (the sort's CF run directions), each output run at its
+  // own position in a temp buffer with 4 words of gap, a descending run
+  // shifted so that b_off = a_off - nb (mod 4) against its A partner.  Passes
+  // >= 2 then run on the persistent TMA/window kernels exactly like the
+  // sort's passes (B bulk-copied straight into its reversed slot).
   if (!temp_bytes || nruns < 0 || (nruns > 0 && !h_run_offsets)) return BCF_ERROR_INVALID_VALUE;
   const bool pairs = d_run_vals != nullptr;
   Params p;
@@ -468,9 +474,10 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   const uint64_t n = nruns > 0 ? h_run_offsets[nruns] : 0;
   for (int r = 0; r < nruns; ++r)
     if (h_run_offsets[r + 1] < h_run_offsets[r] || h_run_offsets[0] != 0) return BCF_ERROR_INVALID_VALUE;
-  const size_t key_bytes = align_up((size_t)n * sizeof(uint32_t), 256);
+  const size_t buf_words = (size_t)n + 4 * ((size_t)nruns + 2) + 64;
+  const size_t key_bytes = align_up(buf_words * sizeof(uint32_t), 256);
   const size_t table_bytes = align_up(sizeof(GroupDesc) * (size_t)(nruns / 2 + 1), 256);
-  const size_t need = 256 + key_bytes * (pairs ? 2 : 1) + table_bytes * 64;
+  const size_t need = 256 + key_bytes * 2 * (pairs ? 2 : 1) + table_bytes * 64;
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -485,46 +492,72 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }
   const Variant& var = launch_table().v[p.E][u_index(p.U)][0][pairs ? 1 : 0];
-  if (!var.merge_table) return BCF_ERROR_UNSUPPORTED;
+  if (!var.merge_table || !var.merge) return BCF_ERROR_UNSUPPORTED;
+  const bool use_tma = var.merge_tma != nullptr && !tma_disabled();
   const long long T = (long long)p.U * p.E;
   char* tb = (char*)align_up((size_t)d_temp, 256);
-  uint32_t* tk = (uint32_t*)tb;
-  uint32_t* tv = pairs ? (uint32_t*)(tb + key_bytes) : nullptr;
-  GroupDesc* dtab = (GroupDesc*)(tb + key_bytes * (pairs ? 2 : 1));
+  uint32_t* tk[2] = {(uint32_t*)tb, (uint32_t*)(tb + key_bytes)};
+  uint32_t* tv[2] = {pairs ? (uint32_t*)(tb + 2 * key_bytes) : nullptr,
+                     pairs ? (uint32_t*)(tb + 3 * key_bytes) : nullptr};
+  GroupDesc* dtab = (GroupDesc*)(tb + key_bytes * 2 * (pairs ? 2 : 1));
   int P = 0;
   while ((1 << P) < nruns) ++P;
-  std::vector<uint64_t> off(h_run_offsets, h_run_offsets + nruns + 1);
-  uint32_t* bk[2] = {d_out, tk};
-  uint32_t* bv[2] = {d_out_vals, tv};
+  struct Run {
+    long long pos, len;
+    int desc;
+  };
+  std::vector<Run> runs(nruns);
+  for (int r = 0; r < nruns; ++r)
+    runs[r] = {(long long)h_run_offsets[r], (long long)(h_run_offsets[r + 1] - h_run_offsets[r]), 0};
   const uint32_t* srck = d_runs;
   const uint32_t* srcv = d_run_vals;
   for (int i = 1; i <= P; ++i) {
-    const int dst = (P - i) % 2;
+    const bool last = i == P;
+    uint32_t* dk = last ? d_out : tk[i & 1];
+    uint32_t* dv = last ? d_out_vals : tv[i & 1];
     std::vector<GroupDesc> tab;
-    std::vector<uint64_t> noff{0};
-    long long tiles = 0;
-    const int nr = (int)off.size() - 1;
-    for (int r = 0; r < nr; r += 2) {
-      GroupDesc g{};
-      g.a_off = (long long)off[r];
-      g.na = (long long)(off[r + 1] - off[r]);
-      g.b_off = (long long)off[std::min(r + 1, nr)];
-      g.nb = r + 1 < nr ? (long long)(off[r + 2] - off[r + 1]) : 0;
-      g.out_off = g.a_off;
-      g.tile_begin = tiles;
-      tiles += (g.na + g.nb + T - 1) / T;
-      noff.push_back(off[std::min(r + 2, nr)]);
-      if (g.na + g.nb > 0) tab.push_back(g);
+    std::vector<Run> next;
+    long long tiles = 0, cursor = 0;
+    const int nr = (int)runs.size();
+    for (int r = 0, g = 0; r < nr; r += 2, ++g) {
+      const Run& A = runs[r];
+      const Run B = r + 1 < nr ? runs[r + 1] : Run{A.pos + A.len, 0, 1};
+      GroupDesc gd{};
+      gd.a_off = A.pos;
+      gd.na = A.len;
+      gd.b_off = B.pos;
+      gd.nb = B.len;
+      gd.b_desc = B.desc;
+      Run o{0, A.len + B.len, 0};
+      if (!last) {
+        o.desc = g & 1;
+        o.pos = cursor;
+        // a descending output (next pass's B) sits at pos = A' pos - len (mod 4)
+        // against its partner A' = the previous group's output
+        if (o.desc) o.pos += (((next.back().pos - o.len - cursor) % 4) + 4) % 4;
+        cursor = o.pos + o.len + 4;
+      }
+      gd.out_off = o.pos;
+      gd.out_desc = o.desc;
+      gd.tile_begin = tiles;
+      tiles += (o.len + T - 1) / T;
+      if (o.len > 0) tab.push_back(gd);
+      next.push_back(o);
     }
     GroupDesc* dt = dtab + (size_t)(i - 1) * (table_bytes / sizeof(GroupDesc));
     cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_fail(e);
-    MergeArgs ma{srck, srcv, bk[dst], bv[dst], (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
-    e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
+    MergeArgs ma{srck, srcv, dk, dv, (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
+    if (i == 1)  // the caller's runs: all ascending
+      e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
+    else if (use_tma)
+      e = launch("merge_runs", n, s, [&] { return var.merge_tma(ma, tiles, s); });
+    else
+      e = launch("merge_runs", n, s, [&] { return var.merge(ma, tiles, s); });
     if (e != cudaSuccess) return cuda_fail(e);
-    srck = bk[dst];
-    srcv = bv[dst];
-    off.swap(noff);
+    srck = dk;
+    srcv = dv;
+    runs.swap(next);
   }
   return BCF_SUCCESS;
 }

@@ -208,6 +208,29 @@ def test_merge_runs_stable(sizes):
     np.testing.assert_array_equal(to_host(k_only), ek)
 
 
+@pytest.mark.parametrize("sizes", [[300001, 299999, 12345, 500000, 7, 250000, 0, 333333],
+                                   [1 << 20] * 4, [123457] * 5, [2, 3, 5, 7, 11, 13, 17]])
+@pytest.mark.parametrize("keyspace", [50, 1 << 32])
+@pytest.mark.parametrize("params", [None, "15x256"])
+def test_merge_runs_large(sizes, keyspace, params):
+    """bcf_merge_runs_u32 at sizes spanning many tiles and CTAs: pass 1 on the
+    plain kernel (ascending runs), later passes on the persistent TMA/window
+    kernels over CF run directions; keys only and pairs."""
+    prm = bcf.make_params(15, 256) if params else None
+    rng = np.random.default_rng(sum(sizes) + keyspace % 97)
+    runs = [np.sort(rng.integers(0, keyspace, size=s, dtype=np.uint64).astype(np.uint32), kind="stable")
+            for s in sizes]
+    keys = np.concatenate(runs)
+    vals = np.arange(keys.size, dtype=np.uint32)
+    offs = np.concatenate([[0], np.cumsum(sizes)]).astype(np.uint64)
+    ek, ev = oracle.sort_pairs_u32(keys, vals)
+    ko = bcf.merge_runs(to_dev(keys), offs, params=prm)
+    np.testing.assert_array_equal(to_host(ko), ek)
+    ko, vo = bcf.merge_runs(to_dev(keys), offs, values=to_dev(vals), params=prm)
+    np.testing.assert_array_equal(to_host(ko), ek)
+    np.testing.assert_array_equal(to_host(vo), ev)
+
+
 MERGE_SIZES = [(0, 0), (0, 5), (7, 0), (1, 1), (3968 * 3 + 17, 5000), (100000, 1), (1, 100000),
                (70001, 70003), (4352, 4352), (1 << 20, (1 << 20) - 3)]
 
