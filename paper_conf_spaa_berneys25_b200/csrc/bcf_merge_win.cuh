@@ -197,6 +197,14 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
         b_lo = align_up4(eb0);
         eb1 = b_lo;
       }
+      // the aligned A range must not run past A's last word (a caller's
+      // array, bcf_merge_u32): its last <= 3 words then come from the edge
+      // lanes instead (after the overlap split, which clips A the same way)
+      if (WA && (long long)a_hi > grp.a_off + grp.na - (oA - c)) {
+        ea1 = c + WA;
+        a_hi = align_dn4(ea1);
+        ea0 = a_hi;
+      }
       uint32_t* sk = stage(s);
       // edge words first (their loads overlap the bulk-copy issue)
       int w = -1;
