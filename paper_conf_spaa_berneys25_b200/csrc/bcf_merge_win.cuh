@@ -41,9 +41,9 @@ __host__ __device__ constexpr int win_stage_words() {
 #define BCF_WIN_STAGES 2
 #endif
 constexpr int WIN_STAGES = BCF_WIN_STAGES;
-template <int E, int U>
+template <int E, int U, bool PAIRS = false>
 __host__ __device__ constexpr size_t win_smem_bytes() {
-  return (size_t)WIN_STAGES * win_stage_words<E, U>() * sizeof(uint32_t);
+  return (size_t)WIN_STAGES * win_stage_words<E, U>() * sizeof(uint32_t) * (PAIRS ? 2 : 1);
 }
 
 struct WinMeta {
@@ -78,13 +78,15 @@ __device__ __forceinline__ int warp_prefix_count(int n, P pred, int lane) {
 }
 
 // resident CTAs per SM the kernel is built for (5 at u = 128)
-template <int U>
+template <int U, bool PAIRS = false>
 __host__ __device__ constexpr int win_min_blocks() {
+  // pairs: twice the stage bytes and a value + tag register per key
+  if (PAIRS) return U <= 128 ? 3 : (U <= 256 ? 2 : 1);
   return WIN_STAGES > 2 ? (U <= 128 ? 3 : 1) : (U <= 128 ? 5 : (U <= 256 ? 2 : 1));
 }
 
-template <int E, int U>
-__global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_kernel(MergeArgs args, long long tiles,
+template <int E, int U, bool PAIRS = false>
+__global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass_win_kernel(MergeArgs args, long long tiles,
                                                                 long long per_cta) {
   constexpr int T = U * E;
   constexpr int S2 = win_span<E, U>();
@@ -106,7 +108,9 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
   long long t_begin, t_end;
   cta_tile_range(tiles, per_cta, t_begin, t_end);
   if (t_end <= t_begin) return;
-  auto stage = [&](int s) { return smem_dyn + (size_t)s * SW; };
+  // stage s: SW key words, then (pairs) SW value words at the same offsets
+  auto stage = [&](int s) { return smem_dyn + (size_t)s * SW * (PAIRS ? 2 : 1); };
+  auto stage_v = [&](int s) { return smem_dyn + (size_t)s * SW * (PAIRS ? 2 : 1) + SW; };
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
@@ -124,6 +128,8 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     const uint32_t* __restrict__ src = args.src_k;
     // B runs (table mode, bcf_merge_u32): a separate base, stored descending
     const uint32_t* __restrict__ srcB = args.src_kb ? args.src_kb : args.src_k;
+    const uint32_t* __restrict__ srcv = args.src_v;
+    const uint32_t* __restrict__ srcvB = args.src_vb ? args.src_vb : args.src_v;
     const long long dst_phase = (long long)(((uintptr_t)args.dst_k >> 2) & 3);
 
     // current segment: the part of one merge group inside this CTA's range
@@ -210,6 +216,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       int w = -1;
       long long gw = 0;
       const uint32_t* __restrict__ esrc = lane >= 4 ? srcB : src;
+      const uint32_t* __restrict__ esrcv = lane >= 4 ? srcvB : srcv;
       if (lane >= 1 && lane <= 3 && ea0 + lane - 1 < ea1) {
         w = ea0 + lane - 1;
         gw = oA + (w - c);
@@ -218,9 +225,15 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
         gw = oB + (w - c);
       }
       if (lane == 0) {
-        tma::mbar_expect_tx(&full_bar[s], (uint32_t)(a_hi + (b_hi - b_lo)) * 4u);
+        tma::mbar_expect_tx(&full_bar[s], (uint32_t)(a_hi + (b_hi - b_lo)) * 4u * (PAIRS ? 2u : 1u));
         if (a_hi > 0) tma::bulk_g2s(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
         if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, srcB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        if constexpr (PAIRS) {
+          uint32_t* sv = stage_v(s);
+          if (a_hi > 0) tma::bulk_g2s(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
+          if (b_hi > b_lo)
+            tma::bulk_g2s(sv + b_lo, srcvB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        }
         // L2 prefetch of the keys the next window will need beyond this one
         // (both runs are consumed sequentially): the next window's bulk loads,
         // issued one subtile later, then hit L2 instead of DRAM
@@ -238,6 +251,10 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       }
       const uint32_t ev = w >= 0 ? __ldg(esrc + gw) : 0u;
       if (w >= 0) sk[w] = ev;
+      if constexpr (PAIRS) {
+        const uint32_t evv = w >= 0 ? __ldg(esrcv + gw) : 0u;
+        if (w >= 0) stage_v(s)[w] = evv;
+      }
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);
     };
@@ -264,8 +281,11 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       const int w0 = M.cout + qlo, w1 = M.cout + qhi;
       int ilo = align_up4(w0), ihi = align_dn4(w1);
       if (lane == 0) {
-        if (ihi > ilo)
+        if (ihi > ilo) {
           tma::bulk_s2g(args.dst_k + (M.c0 - M.cout) + ilo, stage(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
+          if constexpr (PAIRS)
+            tma::bulk_s2g(args.dst_v + (M.c0 - M.cout) + ilo, stage_v(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
+        }
         tma::bulk_commit();
       }
     };
@@ -328,7 +348,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
 
   // ============================ consumers ============================
   const bool decode = args.decode_f32 != 0;
-  uint32_t dummy[E];
+  uint32_t val[E];  // values (pairs); unused for keys
   for (int i = 0;; ++i) {
     const int s = i % S;
     if (tid == 0 && i < 31) BCF_TRACE_AT(1 + 4 * i);
@@ -337,6 +357,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     const WinMeta M = meta[s];
     if (M.exit) break;
     uint32_t* sk = stage(s) + M.c;  // logical index -> sk[index]
+    uint32_t* sv = stage_v(s) + M.c;
     const int WA = M.WA, WB = M.WB, cmax = M.cmax;
     const int D = tid * E;
     const int Dw = warp * W * E;
@@ -390,10 +411,10 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     const int b = Dc - a;
     uint32_t key[E];
     if (cnt == T)
-      dual_subsequence_gather<E, false, true>(sk, sk, 0, S2, a, b, nA, nB, key, dummy, PAD_KEY);
+      dual_subsequence_gather<E, PAIRS, true>(sk, PAIRS ? sv : sk, 0, S2, a, b, nA, nB, key, val, PAD_KEY);
     else
-      dual_subsequence_gather<E, false, false>(sk, sk, 0, S2, a, b, nA, nB, key, dummy, PAD_KEY);
-    merge_registers<E, false>(key, dummy, a, nA, nB);
+      dual_subsequence_gather<E, PAIRS, false>(sk, PAIRS ? sv : sk, 0, S2, a, b, nA, nB, key, val, PAD_KEY);
+    merge_registers<E, PAIRS>(key, val, a, nA, nB);
     if (decode) {
 #pragma unroll
       for (int q = 0; q < E; ++q) key[q] = f32_decode(key[q]);
@@ -401,12 +422,19 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
     tma::named_bar_sync(1, U);  // every consumer has finished reading the stage
     if (tid == 0 && i < 30) BCF_TRACE_AT(160 + 3 * i);
     uint32_t* ok = stage(s) + M.cout;
+    uint32_t* ov = stage_v(s) + M.cout;
     if (M.desc) {
 #pragma unroll
-      for (int q = 0; q < E; ++q) ok[T - E - D + q] = key[E - 1 - q];
+      for (int q = 0; q < E; ++q) {
+        ok[T - E - D + q] = key[E - 1 - q];
+        if constexpr (PAIRS) ov[T - E - D + q] = val[E - 1 - q];
+      }
     } else {
 #pragma unroll
-      for (int q = 0; q < E; ++q) ok[D + q] = key[q];
+      for (int q = 0; q < E; ++q) {
+        ok[D + q] = key[q];
+        if constexpr (PAIRS) ov[D + q] = val[q];
+      }
     }
     tma::fence_proxy_async_smem();  // the producer's bulk store reads these words
     tma::named_bar_sync(1, U);
@@ -423,8 +451,13 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U>()) merge_pass_win_ke
       const uint32_t* sb = stage(s);
       uint32_t* gb = args.dst_k + (M.c0 - M.cout);
       const int nh = ilo - w0, nt = w1 - ihi;  // <= 7, <= 3
-      if (lane < nh) gb[w0 + lane] = sb[w0 + lane];
-      else if (lane >= 8 && lane - 8 < nt) gb[ihi + lane - 8] = sb[ihi + lane - 8];
+      int ew = -1;
+      if (lane < nh) ew = w0 + lane;
+      else if (lane >= 8 && lane - 8 < nt) ew = ihi + lane - 8;
+      if (ew >= 0) {
+        gb[ew] = sb[ew];
+        if constexpr (PAIRS) args.dst_v[(M.c0 - M.cout) + ew] = stage_v(s)[ew];
+      }
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&empty_bar[s]);
     }

@@ -110,18 +110,30 @@ cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int thre
 #ifndef BCF_MERGE_WIN
 #define BCF_MERGE_WIN 1
 #endif
+// BCF_PAIRS_TMA=1: pairs passes on the 3-stage exact-split TMA kernel instead
+// of the window kernel (A/B measurements)
+inline bool pairs_tma_forced() {
+  static const bool on = [] {
+    const char* v = getenv("BCF_PAIRS_TMA");
+    return v && v[0] == '1';
+  }();
+  return on;
+}
+
 template <int E, int U, bool PAIRS>
 cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s) {
   static PersistentCache pc;  // one per (E, U, PAIRS) instantiation
-  // the 2-stage window ring needs 2 x 2T words: beyond 227 KB (E = 31,
-  // u = 512) fall back to the 3-stage exact-split TMA kernel
-  constexpr bool win_fits = win_smem_bytes<E, U>() <= 227 * 1024;
-  if constexpr (!PAIRS && BCF_MERGE_WIN && win_fits) {
-    return launch_persistent(merge_pass_win_kernel<E, U>, pc, win_smem_bytes<E, U>(), U + 32, a, tiles, s);
-  } else {
-    return launch_persistent(merge_pass_tma_kernel<E, U, PAIRS>, pc, tma_smem_bytes<E, U, PAIRS>(), U + 32,
-                             a, tiles, s);
+  // the 2-stage window ring (x2 for pairs) must fit in 227 KB; otherwise the
+  // 3-stage exact-split TMA kernel
+  constexpr bool win_fits = win_smem_bytes<E, U, PAIRS>() <= 227 * 1024;
+  if constexpr (BCF_MERGE_WIN && win_fits) {
+    if (!PAIRS || !pairs_tma_forced())
+      return launch_persistent(merge_pass_win_kernel<E, U, PAIRS>, pc, win_smem_bytes<E, U, PAIRS>(), U + 32, a,
+                               tiles, s);
   }
+  static PersistentCache pc_tma;
+  return launch_persistent(merge_pass_tma_kernel<E, U, PAIRS>, pc_tma, tma_smem_bytes<E, U, PAIRS>(), U + 32, a,
+                           tiles, s);
 }
 
 // the window kernel alone (keys only; bcf_merge_u32 passes B through src_kb,
