@@ -184,7 +184,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             k = si.dup_u32_torch(n, si.config_seed(4), dev)
             v = si.iota_u32_torch(n, dev)
             ko, vo = torch.empty_like(k), torch.empty_like(v)
-            prm = bcf.default_pairs_params()  # pairs default (17, 256)
+            prm = bcf.default_pairs_params()  # pairs default (11, 256)
             run = lambda: bcf.sort_pairs(k, v, ko, vo, params=prm, temp=temp)  # noqa: E731
             workload = "2^26 uint32 (key & 0xFFFF, heavy duplicates) + uint32 value (index) pairs, stable"
         if name.startswith("f32") or name.startswith("merge"):

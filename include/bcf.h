@@ -68,7 +68,7 @@ typedef struct {
 } bcf_params;
 
 /* Default (E, u) chosen for sm_100a by measurement: keys
-   (u32 / f32) (31, 128); pairs (17, 256).  A zero field in the params passed
+   (u32 / f32) (31, 128); pairs (11, 256).  A zero field in the params passed
    to a sort selects that entry point's default. */
 void bcf_default_params(bcf_params* p);
 void bcf_default_pairs_params(bcf_params* p);

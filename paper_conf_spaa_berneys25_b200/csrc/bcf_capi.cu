@@ -51,9 +51,10 @@ LaunchTable& launch_table() {
 static constexpr int DEFAULT_E = 31;
 static constexpr int DEFAULT_U = 128;
 // Pairs carry a value and a tag per register: E = 31 spills the register
-// budget, (17, 256) is the measured best of the pairs sweep at 2^26
-// (profiles/r01_pairs_sweep_2p26.txt: 12.1 G pairs/s vs 7.1 at (31, 128)).
-static constexpr int DEFAULT_E_PAIRS = 17;
+// budget; with pairs merge passes on the window kernel, (11, 256) is the
+// measured best of the pairs sweep at 2^26 (profiles/r01_pairs_sweep_window_2p26.txt:
+// 5.22 ms vs 5.47 at (17, 256), the previous default under the TMA kernel).
+static constexpr int DEFAULT_E_PAIRS = 11;
 static constexpr int DEFAULT_U_PAIRS = 256;
 
 // ---------------------------------------------------------------------------

@@ -53,7 +53,7 @@ def test_default_params():
     assert p.block_threads in (128, 256, 512)
     assert p.algo == bcf.ALGO_CONFLICT_FREE
     q = bcf.default_pairs_params()
-    assert (q.items_per_thread, q.block_threads, q.algo) == (17, 256, bcf.ALGO_CONFLICT_FREE)
+    assert (q.items_per_thread, q.block_threads, q.algo) == (11, 256, bcf.ALGO_CONFLICT_FREE)
 
 
 def _query(fn, n, params=None, pairs=False):
@@ -187,7 +187,8 @@ def test_sort_plan():
     assert bcf.sort_plan(7937)["merge_passes"] == 1
     assert bcf.sort_plan(1 << 24, bcf.make_params(31, 128, bcf.ALGO_BASELINE)) == \
         {"block_sort_tile": 3968, "merge_tile": 3968, "merge_passes": 13}
-    assert bcf.sort_plan(1 << 26, pairs=True) == {"block_sort_tile": 17 * 256, "merge_tile": 17 * 256,
-                                                  "merge_passes": 14}
+    assert bcf.sort_plan(1 << 26, pairs=True) == {"block_sort_tile": 11 * 256, "merge_tile": 11 * 256,
+                                                  "merge_passes": 15}  # ceil(log2(2^26 / 2816))
+    assert bcf.sort_plan(1 << 26, bcf.make_params(17, 256), pairs=True)["merge_passes"] == 14
     assert bcf.sort_plan(1 << 24, bcf.make_params(15, 256)) == {"block_sort_tile": 3840, "merge_tile": 3840,
                                                                "merge_passes": 13}
