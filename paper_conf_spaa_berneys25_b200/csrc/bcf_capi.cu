@@ -228,7 +228,11 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
     uint32_t* dv = i == P ? out_v : ((i & 1) ? YV : XV);
     MergeArgs ma{sk, sv, dk, dv, (long long)n, Tbs << (i - 1), i + lg_bs,
                  (f32 && i == P) ? 1 : 0, cf ? 1 : 0, nullptr, 0, trace_for_pass(i)};
-    if (use_tma)
+    // the persistent kernels bulk-store keys and values at one 16-byte phase
+    // (the keys'): a final pass into key / value outputs of different phases
+    // takes the plain kernel
+    const bool phase_ok = !pairs || i < P || (((uintptr_t)out_k ^ (uintptr_t)out_v) & 15) == 0;
+    if (use_tma && phase_ok)
       e = launch("merge_pass", n, s, [&] { return var.merge_tma(ma, tiles, s); });
     else
       e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
@@ -551,7 +555,7 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     MergeArgs ma{srck, srcv, dk, dv, (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
     if (i == 1)  // the caller's runs: all ascending
       e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
-    else if (use_tma)
+    else if (use_tma && (!pairs || !last || (((uintptr_t)d_out ^ (uintptr_t)d_out_vals) & 15) == 0))
       e = launch("merge_runs", n, s, [&] { return var.merge_tma(ma, tiles, s); });
     else
       e = launch("merge_runs", n, s, [&] { return var.merge(ma, tiles, s); });
@@ -585,7 +589,7 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
   if (st != BCF_SUCCESS) return st;
   if (p.algo != BCF_ALGO_CONFLICT_FREE) return BCF_ERROR_UNSUPPORTED;
   // keys only: room for B reversed (window kernel path), +8 words of phase/tail slack
-  const size_t need = 256 + align_up(sizeof(GroupDesc), 256) + (pairs ? 0 : align_up(4 * ((size_t)nb + 8), 256));
+  const size_t need = 256 + align_up(sizeof(GroupDesc), 256) + align_up(4 * ((size_t)nb + 8), 256) * (pairs ? 2 : 1);
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -611,7 +615,9 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
   g.na = (long long)na;
   g.nb = (long long)nb;
   GroupDesc* dt = (GroupDesc*)align_up((size_t)d_temp, 256);
-  if (!pairs && var.merge_win && ((uintptr_t)d_a & 15) == 0 && !tma_disabled()) {
+  const bool win_ok = var.merge_win && ((uintptr_t)d_a & 15) == 0 && !tma_disabled() &&
+                      (!pairs || (((uintptr_t)d_a_vals & 15) == 0 && (((uintptr_t)d_out ^ (uintptr_t)d_out_vals) & 15) == 0));
+  if (win_ok) {
     // persistent window kernel (0.8 of HBM per pass at 2^28): B reversed into
     // temp at word phase b_off = -nb mod 4, so that A's and B's windows share
     // one 16-byte phase (a_off - b_off - nb = 0 mod 4, as in the sort's passes)
@@ -626,7 +632,15 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
       return cudaGetLastError();
     });
     if (e != cudaSuccess) return cuda_fail(e);
-    MergeArgs ma{d_a, nullptr, d_out, nullptr, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, rb, nullptr};
+    uint32_t* rbv = pairs ? rb + align_up(4 * ((size_t)nb + 8), 256) / 4 : nullptr;
+    if (pairs) {
+      e = launch("merge_reverse", nb, s, [&] {
+        reverse_u32_kernel<<<(unsigned)blocks, 256, 0, s>>>(d_b_vals, rbv + g.b_off, (long long)nb);
+        return cudaGetLastError();
+      });
+      if (e != cudaSuccess) return cuda_fail(e);
+    }
+    MergeArgs ma{d_a, d_a_vals, d_out, d_out_vals, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, rb, rbv};
     e = launch("merge", n, s, [&] { return var.merge_win(ma, tiles, s); });
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }

@@ -138,10 +138,11 @@ cudaError_t launch_merge_tma(const MergeArgs& a, long long tiles, cudaStream_t s
 
 // the window kernel alone (keys only; bcf_merge_u32 passes B through src_kb,
 // which only the window and plain kernels read)
-template <int E, int U>
+template <int E, int U, bool PAIRS>
 cudaError_t launch_merge_win(const MergeArgs& a, long long tiles, cudaStream_t s) {
   static PersistentCache pc;
-  return launch_persistent(merge_pass_win_kernel<E, U>, pc, win_smem_bytes<E, U>(), U + 32, a, tiles, s);
+  return launch_persistent(merge_pass_win_kernel<E, U, PAIRS>, pc, win_smem_bytes<E, U, PAIRS>(), U + 32, a, tiles,
+                           s);
 }
 
 template <int E, int U>
@@ -157,7 +158,9 @@ void register_eu(LaunchTable& t) {
     t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
     t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;
     if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
-      t.v[E][ui][0][0].merge_win = &launch_merge_win<E, U>;
+      t.v[E][ui][0][0].merge_win = &launch_merge_win<E, U, false>;
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
+      t.v[E][ui][0][1].merge_win = &launch_merge_win<E, U, true>;
   }
 }
 

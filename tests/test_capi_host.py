@@ -112,7 +112,7 @@ def test_merge_u32_query_and_validation():
     tbp = ctypes.c_size_t(0)
     fake0 = ctypes.c_void_p(4096)
     assert L.bcf_merge_u32(None, 100, None, 100, fake0, fake0, None, fake0, None, ctypes.byref(tbp), None,
-                           None) == 0 and 0 < tbp.value <= 1024
+                           None) == 0 and 0 < tbp.value <= 512 + 2 * 768
     assert L.bcf_merge_u32(None, 1, None, 1, None, None, None, None, None, None, None,
                            None) == bcf.BCF_ERROR_INVALID_VALUE
     small = ctypes.c_size_t(need - 1)

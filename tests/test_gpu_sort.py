@@ -170,6 +170,38 @@ def test_in_place_and_unaligned():
         assert int(dst_big[0]) == 0 and int(dst_big[n + 3]) == 0  # no writes outside
 
 
+@pytest.mark.parametrize("n", [3000, 200001, 1 << 20])
+def test_pairs_unaligned_mismatched_phases(n):
+    """Key and value buffers at different 16-byte phases (inputs and outputs):
+    the persistent kernels' bulk stores assume one phase, so such a final pass
+    must take the plain kernel; sort_pairs, merge_runs and merge stay exact."""
+    k = si.dup_u32(n, si.config_seed(4) + n)
+    v = si.iota_u32(n)
+    ek, ev = oracle.sort_pairs_u32(k, v)
+
+    def view(x, off):
+        big = torch.zeros(x.size + 4, dtype=torch.int32, device=DEV)
+        t = big[off:off + x.size]
+        t.copy_(to_dev(x))
+        return t
+
+    kin, vin = view(k, 1), view(v, 2)
+    kout, vout = view(np.zeros(n, np.uint32), 3), view(np.zeros(n, np.uint32), 0)
+    bcf.sort_pairs(kin, vin, kout, vout)
+    np.testing.assert_array_equal(to_host(kout), ek)
+    np.testing.assert_array_equal(to_host(vout), ev)
+    # two sorted halves -> merge (pairs), outputs at different phases
+    h = n // 2
+    ak, av = oracle.sort_pairs_u32(k[:h], v[:h])
+    bk, bv = oracle.sort_pairs_u32(k[h:], v[h:])
+    mk, mv = oracle.sort_pairs_u32(np.concatenate([ak, bk]), np.concatenate([av, bv]))
+    for aoff, ooff in ((0, 0), (1, 2), (0, 3)):
+        ko, vo = view(np.zeros(n, np.uint32), ooff), view(np.zeros(n, np.uint32), 0)
+        bcf.merge(view(ak, aoff), view(bk, 0), view(av, 0), view(bv, 1), out=ko, out_values=vo)
+        np.testing.assert_array_equal(to_host(ko), mk)
+        np.testing.assert_array_equal(to_host(vo), mv)
+
+
 def test_input_untouched():
     x = si.uniform_u32(50000, 5)
     t = to_dev(x)
