@@ -250,10 +250,19 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
       }
       const uint32_t ev = w >= 0 ? __ldg(esrc + gw) : 0u;
-      if (w >= 0) sk[w] = ev;
-      if constexpr (PAIRS) {
-        const uint32_t evv = w >= 0 ? __ldg(esrcv + gw) : 0u;
-        if (w >= 0) stage_v(s)[w] = evv;
+      const uint32_t evv = (PAIRS && w >= 0) ? __ldg(esrcv + gw) : 0u;
+      // lane 0 stores the <= 6 edge words itself, then release-arrives: the
+      // stores precede the arrive in one thread's program order (a lane-l
+      // store ordered only through __syncwarp is invisible to racecheck)
+#pragma unroll
+      for (int l = 1; l <= 6; ++l) {
+        const int wl = __shfl_sync(FULL, w, l);
+        const uint32_t kl = __shfl_sync(FULL, ev, l);
+        const uint32_t vl = PAIRS ? __shfl_sync(FULL, evv, l) : 0u;
+        if (lane == 0 && wl >= 0) {
+          sk[wl] = kl;
+          if constexpr (PAIRS) stage_v(s)[wl] = vl;
+        }
       }
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);
