@@ -459,6 +459,13 @@ bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint
   return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
 }
 
+// B reversed into temp for the window kernel, whose bulk copies need B
+// stored descending (element y of B at out[nb-1-y])
+__global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, long long n) {
+  for (long long j = blockIdx.x * (long long)blockDim.x + threadIdx.x; j < n; j += (long long)gridDim.x * blockDim.x)
+    out[j] = __ldg(in + (n - 1 - j));
+}
+
 bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals, const uint64_t* h_run_offsets,
                               int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals, void* d_temp,
                               size_t* temp_bytes, const bcf_params* pp, void* stream) {
@@ -482,7 +489,8 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   const size_t buf_words = (size_t)n + 4 * ((size_t)nruns + 2) + 64;
   const size_t key_bytes = align_up(buf_words * sizeof(uint32_t), 256);
   const size_t table_bytes = align_up(sizeof(GroupDesc) * (size_t)(nruns / 2 + 1), 256);
-  const size_t need = 256 + key_bytes * 2 * (pairs ? 2 : 1) + table_bytes * 64;
+  // + one buffer (per array) for the odd runs reversed before pass 1
+  const size_t need = 256 + key_bytes * 3 * (pairs ? 2 : 1) + table_bytes * 64;
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -504,7 +512,9 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   uint32_t* tk[2] = {(uint32_t*)tb, (uint32_t*)(tb + key_bytes)};
   uint32_t* tv[2] = {pairs ? (uint32_t*)(tb + 2 * key_bytes) : nullptr,
                      pairs ? (uint32_t*)(tb + 3 * key_bytes) : nullptr};
-  GroupDesc* dtab = (GroupDesc*)(tb + key_bytes * 2 * (pairs ? 2 : 1));
+  uint32_t* rk = (uint32_t*)(tb + key_bytes * (pairs ? 4 : 2));  // reversed odd runs
+  uint32_t* rv = pairs ? (uint32_t*)(tb + key_bytes * 5) : nullptr;
+  GroupDesc* dtab = (GroupDesc*)(tb + key_bytes * 3 * (pairs ? 2 : 1));
   int P = 0;
   while ((1 << P) < nruns) ++P;
   struct Run {
@@ -514,6 +524,32 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   std::vector<Run> runs(nruns);
   for (int r = 0; r < nruns; ++r)
     runs[r] = {(long long)h_run_offsets[r], (long long)(h_run_offsets[r + 1] - h_run_offsets[r]), 0};
+  // Pass 1 on the window kernel too: the odd (B) runs reversed into rk
+  // (+8 B per B key), each at word phase A pos - len (mod 4) against its A
+  // partner, read through src_kb / src_vb; A straight from the caller's
+  // 16-byte aligned runs.  Bounded run count (one reverse launch per B run).
+  const bool rev1 = var.merge_win != nullptr && !tma_disabled() && nruns <= 64 &&
+                    ((uintptr_t)d_runs & 15) == 0 &&
+                    (!pairs || (((uintptr_t)d_run_vals & 15) == 0 &&
+                                (P > 1 || (((uintptr_t)d_out ^ (uintptr_t)d_out_vals) & 15) == 0)));
+  if (rev1) {
+    long long cur = 0;
+    for (int r = 1; r < nruns; r += 2) {
+      const long long len = runs[r].len;
+      const long long pos = cur + ((((runs[r - 1].pos - len - cur) % 4) + 4) % 4);
+      cur = pos + len + 8;
+      runs[r] = {pos, len, 1};
+      if (len == 0) continue;
+      const long long src0 = (long long)h_run_offsets[r];
+      const long long blocks = std::min<long long>((len + 255) / 256, 148LL * 16);
+      cudaError_t e = launch("merge_reverse", (uint64_t)len, s, [&] {
+        reverse_u32_kernel<<<(unsigned)blocks, 256, 0, s>>>(d_runs + src0, rk + pos, len);
+        if (pairs) reverse_u32_kernel<<<(unsigned)blocks, 256, 0, s>>>(d_run_vals + src0, rv + pos, len);
+        return cudaGetLastError();
+      });
+      if (e != cudaSuccess) return cuda_fail(e);
+    }
+  }
   const uint32_t* srck = d_runs;
   const uint32_t* srcv = d_run_vals;
   for (int i = 1; i <= P; ++i) {
@@ -553,7 +589,11 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_fail(e);
     MergeArgs ma{srck, srcv, dk, dv, (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
-    if (i == 1)  // the caller's runs: all ascending
+    if (i == 1 && rev1) {
+      ma.src_kb = rk;
+      ma.src_vb = rv;
+      e = launch("merge_runs", n, s, [&] { return var.merge_win(ma, tiles, s); });
+    } else if (i == 1)  // the caller's runs: all ascending
       e = launch("merge_runs", n, s, [&] { return var.merge_table(ma, tiles, s); });
     else if (use_tma && (!pairs || !last || (((uintptr_t)d_out ^ (uintptr_t)d_out_vals) & 15) == 0))
       e = launch("merge_runs", n, s, [&] { return var.merge_tma(ma, tiles, s); });
@@ -565,13 +605,6 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
     runs.swap(next);
   }
   return BCF_SUCCESS;
-}
-
-// B reversed into temp for the window kernel, whose bulk copies need B
-// stored descending (element y of B at out[nb-1-y])
-__global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, long long n) {
-  for (long long j = blockIdx.x * (long long)blockDim.x + threadIdx.x; j < n; j += (long long)gridDim.x * blockDim.x)
-    out[j] = __ldg(in + (n - 1 - j));
 }
 
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
