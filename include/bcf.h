@@ -161,9 +161,10 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
    LSU-staged CF kernel reading B ascending.  Temp (CUB-style query): 512
    bytes (group descriptor), + 4 (nb + 8) bytes (rounded up to 256) for keys
    only.  na = nb = 0 is a no-op; one side empty is a device copy.  Only
-   BCF_ALGO_CONFLICT_FREE.  Like bcf_merge_runs_u32 it stages its group
-   descriptor(s) with a stream-ordered H2D copy from pageable host memory, so
-   (unlike the sorts) it cannot be captured into a CUDA graph. */
+   BCF_ALGO_CONFLICT_FREE.  Kernel launches only (the group descriptor is
+   written by a 1-thread kernel), so the call can be captured into a CUDA
+   graph, like the sorts; bcf_merge_runs_u32 stages its descriptor table with
+   a pageable H2D copy and cannot. */
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
                          const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
                          uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* p,

@@ -459,6 +459,11 @@ bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint
   return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
 }
 
+// the one group descriptor of bcf_merge_u32, written by a 1-thread kernel
+// (a kernel parameter, not a pageable H2D copy: the call stays capturable
+// into a CUDA graph)
+__global__ void write_desc_kernel(GroupDesc* d, GroupDesc g) { *d = g; }
+
 // B reversed into temp for the window kernel, whose bulk copies need B
 // stored descending (element y of B at out[nb-1-y])
 __global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, long long n) {
@@ -657,7 +662,8 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
     uint32_t* rb = (uint32_t*)((char*)dt + align_up(sizeof(GroupDesc), 256));
     g.b_off = (long long)((4 - (nb & 3)) & 3);
     g.b_desc = 1;
-    cudaError_t e = cudaMemcpyAsync(dt, &g, sizeof(g), cudaMemcpyHostToDevice, s);
+    write_desc_kernel<<<1, 1, 0, s>>>(dt, g);
+    cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e);
     const long long blocks = std::min<long long>((long long)((nb + 255) / 256), 148LL * 16);
     e = launch("merge_reverse", nb, s, [&] {
@@ -677,8 +683,8 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
     e = launch("merge", n, s, [&] { return var.merge_win(ma, tiles, s); });
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }
-  // pageable source: cudaMemcpyAsync returns once `g` has been staged
-  cudaError_t e = cudaMemcpyAsync(dt, &g, sizeof(g), cudaMemcpyHostToDevice, s);
+  write_desc_kernel<<<1, 1, 0, s>>>(dt, g);
+  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e);
   MergeArgs ma{d_a, d_a_vals, d_out, d_out_vals, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, d_b, d_b_vals};
   e = launch("merge", n, s, [&] { return var.merge_table(ma, tiles, s); });

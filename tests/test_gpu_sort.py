@@ -202,6 +202,38 @@ def test_pairs_unaligned_mismatched_phases(n):
         np.testing.assert_array_equal(to_host(vo), mv)
 
 
+def test_cuda_graph_capture_sort_and_merge():
+    """The sort and bcf_merge_u32 are kernel launches only: captured once into
+    a CUDA graph, each replay re-sorts / re-merges the current buffer contents."""
+    n = (1 << 20) + 17
+    x = to_dev(si.uniform_u32(n, 11))
+    out = torch.empty_like(x)
+    temp = bcf.temp_buffer(n, device=DEV)
+    a0 = np.sort(si.uniform_u32(70001, 12))
+    b0 = np.sort(si.uniform_u32(50003, 13))
+    a, b = to_dev(a0), to_dev(b0)
+    mo = torch.empty(a.numel() + b.numel(), dtype=torch.int32, device=DEV)
+    mtemp = bcf.merge_temp(a.numel(), b.numel(), device=DEV)
+    bcf.sort(x, out=out, temp=temp)  # warm-up outside the capture (attribute caches)
+    bcf.merge(a, b, out=mo, temp=mtemp)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        bcf.sort(x, out=out, temp=temp)
+        bcf.merge(a, b, out=mo, temp=mtemp)
+    for seed in (21, 22):
+        xs = si.uniform_u32(n, seed)
+        x.copy_(to_dev(xs))
+        a1 = np.sort(si.uniform_u32(70001, seed + 100))
+        b1 = np.sort(si.uniform_u32(50003, seed + 200))
+        a.copy_(to_dev(a1))
+        b.copy_(to_dev(b1))
+        g.replay()
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(to_host(out), oracle.sort_u32(xs))
+        np.testing.assert_array_equal(to_host(mo), oracle.sort_u32(np.concatenate([a1, b1])))
+
+
 def test_input_untouched():
     x = si.uniform_u32(50000, 5)
     t = to_dev(x)
