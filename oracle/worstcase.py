@@ -12,16 +12,30 @@ Per subproblem of w/d threads and wE/d outputs:
     T: steps (1)-(3), PAPER.md:261-266 (garbled text read per SURVEY.md c7)
 Theorem 8 (combined :342).
 
+Order inside a mixed thread (reading c9): the thread of S-tuple i
+reads its x_i part first and its y_i part last.  The proof
+counts conflicts in the bottom E banks: every column of w words is
+x_i | y_{i+1} | pure tuples (x_i + y_{i+1} = r or E + r, Lemma 7), so a y part
+that ends the column at bank w-1 is in lockstep with the pure threads' scan of
+banks w-E..w-1 only if it is read LAST, and an x part (banks 0..x_i-1, the
+"(x_i - r) misaligned elements") can never be.  Under this order the number of
+reads that land in the scanned bank w-E+s-1 at serial-merge step s is exactly
+Theorem 8 for every 1 < E <= w (tests/test_oracle_worstcase.py); the total
+conflicts are >= Theorem 8, because the x parts, which the proof does not
+count, are read in lockstep with one another.
+
 Multi-level composition (reading c10): start from the sorted output 0..n-1 and
 walk the merge levels top-down; every REGULAR merge group (full, and its run
 size a multiple of wE, i.e. at least two warps of outputs) labels each output
-A or B from T (even subproblem index) / switched T (odd index), with mixed
-threads taking their B members first under T and their A members first under
-switched T (reading c9); every other group gets exactly |A| A-labels at the
-positions with the smallest (h, position) keys of a counter-based stream.
-Labelled positions are stable-partitioned into the two child runs.  At the
-bottom each run of E (one thread's items) is shuffled (Fisher-Yates driven by
-the same counter-based stream) because thread-local order is irrelevant.
+A or B from T (even subproblem index) / switched T (odd index).  Every other
+group (block-sort levels with groups of less than two warps, ragged tails)
+gets a random exact-count labelling that is a closed form of the position: the
+first 2 nb outputs form pairs (2k, 2k+1), pair k is (B, A) if the top bit of a
+counter-based stream word at the pair's absolute index is set and (A, B)
+otherwise, and the remaining na - nb outputs are A.  Labelled positions are
+stable-partitioned into the two child runs.  At the bottom each run of E (one
+thread's items) is shuffled (Fisher-Yates driven by the same counter-based
+stream) because thread-local order is irrelevant.
 """
 from __future__ import annotations
 
@@ -88,8 +102,15 @@ def S_sequence(w: int, E: int):
 
 
 def T_sequence(w: int, E: int):
+    """[(a, b)] of T_sequence_indexed (the S index dropped)."""
+    return [(a, b) for (a, b, _) in T_sequence_indexed(w, E)]
+
+
+def T_sequence_indexed(w: int, E: int):
     """The tuple sequence T of Section 4, |T| = w/d.
 
+    Each entry is (a, b, i): i is the index of the S-tuple it came from, or 0
+    for an inserted pure tuple ((E, 0) / (0, E)).
     E | w (d = E, S empty) is not spelled out by the paper; reading c8 takes
     T = q tuples (E, 0)."""
     assert 1 < E <= w
@@ -97,26 +118,26 @@ def T_sequence(w: int, E: int):
     q, r = euclid(w, E)
     Ed = E // d
     if Ed == 1:
-        return [(E, 0)] * q
+        return [(E, 0, 0)] * q
     S = S_sequence(w, E)
     x = {i: xi for (i, _, xi, _, _, _) in S}
     y = {i: yi for (i, _, _, yi, _, _) in S}
     ab = {i: (a, b) for (i, _, _, _, a, b) in S}
     T = []
     # (1) (a_1, b_1) = (y_1, x_1) = (r, E - r), followed by q tuples of (E, 0)
-    T.append((y[1], x[1]))
-    T.extend([(E, 0)] * q)
+    T.append((y[1], x[1], 1))
+    T.extend([(E, 0, 0)] * q)
     # (2) for i = 1..E/d-2: insert (a_{i+1}, b_{i+1}), then q or q-1 pure tuples
     for i in range(1, Ed - 1):
-        T.append(ab[i + 1])
-        pure = (E, 0) if i % 2 == 0 else (0, E)
+        T.append(ab[i + 1] + (i + 1,))
+        pure = (E, 0, 0) if i % 2 == 0 else (0, E, 0)
         if x[i] + y[i + 1] == r:
             T.extend([pure] * q)
         else:
             assert x[i] + y[i + 1] == E + r  # Lemma 7
             T.extend([pure] * (q - 1))
     # (3) q tuples of (E, 0) if E/d - 1 is even, else (0, E)
-    T.extend([(E, 0) if (Ed - 1) % 2 == 0 else (0, E)] * q)
+    T.extend([(E, 0, 0) if (Ed - 1) % 2 == 0 else (0, E, 0)] * q)
     assert len(T) == w // d
     return T
 
@@ -160,17 +181,28 @@ def warp_thread_tuples(w: int, E: int, first_subproblem_index: int = 0):
 # Multi-level composition (reading c10)
 # ---------------------------------------------------------------------------
 
+def thread_labels(a: int, b: int, i: int, switched_: bool):
+    """Labels (True = B) of one thread's E outputs in merge order (reading c9).
+
+    S-tuple i is (a_i, b_i) = (y_i, x_i) for odd i and (x_i, y_i) for even i
+    (PAPER.md:229-231), so its x part is the B part under T for odd i and the
+    A part for even i; a switched subproblem swaps the lists.
+    The x part is read first, the y part last.  Pure tuples have one list."""
+    if i == 0:
+        return [True] * b + [False] * a
+    x_is_B = (i % 2 == 1) != switched_
+    if x_is_B:
+        return [True] * b + [False] * a
+    return [False] * a + [True] * b
+
+
 def subproblem_label_patterns(w: int, E: int):
     """Label (True = B) of each output position of a T-subproblem and of a
-    switched-T subproblem; mixed threads: B-first under T, A-first under
-    switched T (reading c9)."""
-    T = T_sequence(w, E)
-    Ts = switched(T)
+    switched-T subproblem."""
     pT, pS = [], []
-    for (a, b) in T:
-        pT.extend([True] * b + [False] * a)
-    for (a, b) in Ts:
-        pS.extend([False] * a + [True] * b)
+    for (a, b, i) in T_sequence_indexed(w, E):
+        pT.extend(thread_labels(a, b, i, False))
+        pS.extend(thread_labels(b, a, i, True))
     return np.array(pT, dtype=bool), np.array(pS, dtype=bool)
 
 
@@ -216,17 +248,14 @@ def worst_case_input(n: int, E: int, u: int, seed: int, w: int = 32) -> np.ndarr
             label_B[regular] = np.where(sub % 2 == 0, patT[off], patS[off])
         irr = ~regular
         if irr.any():
+            # pairs (2k, 2k+1) of the first 2 nb outputs: (B, A) if the top bit
+            # of h(absolute pair index) is set, else (A, B); the rest are A
             seed_l = (seed + R * LEVEL_SALT) & MASK64
-            ip = pos[irr]
-            h = stream_np(seed_l, ip)
-            ig = g[irr]
-            order = np.lexsort((ip, h, ig))      # by group, then h, then position
-            sg = ig[order]
-            first = np.searchsorted(sg, sg, side="left")
-            rank = np.arange(len(order)) - first
-            lab = np.empty(len(order), dtype=bool)
-            lab[order] = rank >= na[irr][order]
-            label_B[irr] = lab
+            pi = p[irr]
+            nb = (m - na)[irr]
+            pair_abs = (g0[irr] + pi - (pi & 1)) // 2
+            bit = (stream_np(seed_l, pair_abs) >> np.uint64(63)).astype(np.int64)
+            label_B[irr] = (pi < 2 * nb) & (((pi & 1) ^ bit) == 1)
         key = g * 2 + label_B.astype(np.int64)
         vals = vals[np.argsort(key, kind="stable")]
     # bottom: shuffle every run of E (one thread's items); Fisher-Yates with
