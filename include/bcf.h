@@ -17,7 +17,6 @@
  *    *temp_bytes, then call again with a buffer of at least that size.
  *  - All device work is enqueued on `stream` (may be 0 = legacy default
  *    stream) and is asynchronous; nothing synchronizes the host, except
- *    bcf_worst_case_u32 (host-built input, copied with a synchronous H2D) and
  *    bcf_profile_collect.
  *  - Argument errors are returned synchronously before any launch.
  *    n > 0 with a NULL data pointer -> BCF_ERROR_INVALID_VALUE; a temp buffer
@@ -116,10 +115,14 @@ bcf_status bcf_sort_pairs_u32(const uint32_t* d_keys_in, uint32_t* d_keys_out,
                               void* d_temp, size_t* temp_bytes, const bcf_params* p, void* stream);
 
 /* Worst-case input for the unmodified Thrust mergesort with parameters
-   (E, u) (Section 4: sequences S and T, Theorem 8;
-   multi-level composition per DESIGN.md reading c10).  Writes a permutation
-   of 0..n-1 to d_out.  Deterministic in (n, E, u, seed).  Host-built, then a
-   synchronous copy to the device (off the timed path).  E in [2, 32]. */
+   (E, u) (Section 4: sequences S and T, Theorem 8; inside a
+   mixed thread the x part is read first and the y part last, DESIGN.md
+   reading c9; multi-level composition per reading c10).  Writes a
+   permutation of 0..n-1 to d_out.  Deterministic in (n, E, u, seed).
+   Generated on the device as a closed form of the position (one thread per
+   run of E keys walks the merge levels up), stream-ordered, no host sync, no
+   host memory: any n up to 2^36.  E in [2, 32], u a power of two >= 32;
+   otherwise BCF_ERROR_UNSUPPORTED. */
 bcf_status bcf_worst_case_u32(uint32_t* d_out, uint64_t n, int32_t E, int32_t u, uint64_t seed,
                               void* stream);
 /* Same construction into host memory (no CUDA call). */

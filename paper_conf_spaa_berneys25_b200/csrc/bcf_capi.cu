@@ -18,7 +18,8 @@
 
 namespace bcf {
 namespace wc {
-void generate(uint32_t* out, uint64_t n, int E, int u, uint64_t seed);
+bool generate_host(uint32_t* out, uint64_t n, int E, int u, uint64_t seed);
+cudaError_t generate_device(uint32_t* out, uint64_t n, int E, int u, uint64_t seed, cudaStream_t s, bool* ok);
 }
 
 // ---------------------------------------------------------------------------
@@ -415,33 +416,29 @@ bcf_status bcf_sort_pairs_u32(const uint32_t* d_keys_in, uint32_t* d_keys_out, c
                    (cudaStream_t)stream, false, true);
 }
 
+static bool worst_case_params_ok(uint64_t n, int32_t E, int32_t u) {
+  // merge levels R = E * 2^e need u a power of two; the closed form's small
+  // divisions are exact below 2^40 keys
+  return E >= 2 && E <= 32 && u >= 32 && (u & (u - 1)) == 0 && n <= (1ull << 36);
+}
+
 bcf_status bcf_worst_case_u32_host(uint32_t* h_out, uint64_t n, int32_t E, int32_t u, uint64_t seed) {
   if (n > 0 && !h_out) return BCF_ERROR_INVALID_VALUE;
-  if (E < 2 || E > 32 || u < 32 || u % 32 != 0) return BCF_ERROR_UNSUPPORTED;
-  try {
-    wc::generate(h_out, n, E, u, seed);
-  } catch (...) {
-    return BCF_ERROR_INVALID_VALUE;
-  }
-  return BCF_SUCCESS;
+  if (!worst_case_params_ok(n, E, u)) return BCF_ERROR_UNSUPPORTED;
+  return wc::generate_host(h_out, n, E, u, seed) ? BCF_SUCCESS : BCF_ERROR_UNSUPPORTED;
 }
 
 bcf_status bcf_worst_case_u32(uint32_t* d_out, uint64_t n, int32_t E, int32_t u, uint64_t seed,
                               void* stream) {
   if (n > 0 && !d_out) return BCF_ERROR_INVALID_VALUE;
-  if (E < 2 || E > 32 || u < 32 || u % 32 != 0) return BCF_ERROR_UNSUPPORTED;
+  if (!worst_case_params_ok(n, E, u)) return BCF_ERROR_UNSUPPORTED;
   if (n == 0) return BCF_SUCCESS;
-  uint32_t* h = nullptr;
-  cudaError_t e = cudaMallocHost(&h, n * sizeof(uint32_t));
+  bool ok = true;
+  cudaError_t e = launch("worst_case", n, (cudaStream_t)stream, [&] {
+    return wc::generate_device(d_out, n, E, u, seed, (cudaStream_t)stream, &ok);
+  });
   if (e != cudaSuccess) return cuda_fail(e);
-  bcf_status st = bcf_worst_case_u32_host(h, n, E, u, seed);
-  if (st == BCF_SUCCESS) {
-    e = cudaMemcpyAsync(d_out, h, n * sizeof(uint32_t), cudaMemcpyHostToDevice, (cudaStream_t)stream);
-    if (e == cudaSuccess) e = cudaStreamSynchronize((cudaStream_t)stream);
-    if (e != cudaSuccess) st = cuda_fail(e);
-  }
-  cudaFreeHost(h);
-  return st;
+  return ok ? BCF_SUCCESS : BCF_ERROR_UNSUPPORTED;
 }
 
 bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint32_t* d_pivots, int32_t npiv,

@@ -140,7 +140,8 @@ def test_merge_u32_query_and_validation():
     (15, 64, 15 * 2 ** 9, 1234), (17, 64, 17 * 2 ** 9, 5), (16, 64, 2 ** 13, 7), (12, 64, 12 * 2 ** 9, 9),
     (8, 128, 2 ** 13, 11), (15, 256, 100000, 3), (16, 256, 2 ** 16, 0xB2000000), (9, 128, 7777, 1),
     (13, 512, 1, 2), (7, 128, 0, 3), (15, 512, 15 * 2 ** 14, 4), (11, 256, 50001, 8),
-    (31, 128, 31 * 2 ** 12, 6), (31, 128, 100001, 7),
+    (31, 128, 31 * 2 ** 12, 6), (31, 128, 100001, 7), (19, 64, 19 * 2 ** 10, 12), (24, 128, 24 * 2 ** 11, 13),
+    (32, 64, 2 ** 14 + 3, 14), (2, 32, 5000, 15), (31, 256, 31 * 2 ** 13 + 17, 16),
 ])
 def test_host_worst_case_matches_oracle(E, u, n, seed):
     got = bcf.worst_case_host(n, E, u, seed)
@@ -152,6 +153,13 @@ def test_host_worst_case_is_permutation_at_bench_size():
     n = 1 << 22
     x = bcf.worst_case_host(n, 16, 256, 0xB2000001)
     assert np.array_equal(np.sort(x), np.arange(n, dtype=np.uint32))
+
+
+def test_host_worst_case_matches_oracle_at_the_bench_configuration():
+    """BASELINE configs[1]: 2^24 keys for the default (E, u) = (31, 128)."""
+    n = 1 << 24
+    np.testing.assert_array_equal(bcf.worst_case_host(n, 31, 128, 0xB2000001),
+                                  wc.worst_case_input(n, 31, 128, 0xB2000001))
 
 
 def test_host_batch_query_and_validation():

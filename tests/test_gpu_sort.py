@@ -242,7 +242,8 @@ def test_input_untouched():
 
 
 def test_worst_case_device_matches_oracle():
-    for (E, u, n) in [(16, 256, 1 << 16), (15, 256, 15 * 2 ** 12), (17, 256, 100000)]:
+    for (E, u, n) in [(16, 256, 1 << 16), (15, 256, 15 * 2 ** 12), (17, 256, 100000), (31, 128, 1 << 22),
+                      (31, 128, 31 * 2 ** 15 + 7), (24, 64, 24 * 2 ** 12), (2, 32, 999)]:
         t = bcf.worst_case(n, E, u, seed=42, device=DEV)
         from oracle import worstcase as wc
         np.testing.assert_array_equal(to_host(t), wc.worst_case_input(n, E, u, 42))
