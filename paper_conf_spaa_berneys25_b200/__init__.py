@@ -154,6 +154,15 @@ def _require_cuda(t, name):
         raise BcfError(f"{name} must have 4-byte elements")
 
 
+def _require_out(t, name, n, device):
+    """An output tensor: CUDA, contiguous, 4-byte, n elements on `device`."""
+    _require_cuda(t, name)
+    if t.numel() != n:
+        raise BcfError(f"{name} must hold {n} elements, has {t.numel()}")
+    if t.device != device:
+        raise BcfError(f"{name} is on {t.device}, expected {device}")
+
+
 def _stream(t):
     torch = _torch()
     return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
@@ -185,7 +194,7 @@ def sort(keys, out=None, params: Params | None = None, temp=None):
     n = keys.numel()
     if out is None:
         out = torch.empty_like(keys)
-    _require_cuda(out, "out")
+    _require_out(out, "out", n, keys.device)
     is_f32 = keys.dtype == torch.float32
     fn = lib().bcf_sort_f32 if is_f32 else lib().bcf_sort_u32
     tb = ctypes.c_size_t(0)
@@ -207,8 +216,12 @@ def sort_pairs(keys, values, keys_out=None, values_out=None, params: Params | No
     n = keys.numel()
     if values.numel() != n:
         raise BcfError("keys and values differ in length")
+    if values.device != keys.device:
+        raise BcfError("keys and values are on different devices")
     keys_out = torch.empty_like(keys) if keys_out is None else keys_out
     values_out = torch.empty_like(values) if values_out is None else values_out
+    _require_out(keys_out, "keys_out", n, keys.device)
+    _require_out(values_out, "values_out", n, keys.device)
     tb = ctypes.c_size_t(0)
     pp = ctypes.byref(params) if params is not None else None
     L = lib()
@@ -293,6 +306,10 @@ def merge_runs(runs, run_offsets, values=None, params: Params | None = None):
     _require_cuda(runs, "runs")
     offs = np.ascontiguousarray(np.asarray(run_offsets, dtype=np.uint64))
     nruns = len(offs) - 1
+    if nruns < 0 or int(offs[0]) != 0 or int(offs[-1]) != runs.numel() or np.any(np.diff(offs.astype(np.int64)) < 0):
+        raise BcfError("run_offsets must start at 0, be non-decreasing and end at runs.numel()")
+    if values is not None:
+        _require_out(values, "values", runs.numel(), runs.device)
     out = torch.empty_like(runs)
     out_v = torch.empty_like(values) if values is not None else None
     L = lib()
@@ -334,8 +351,15 @@ def merge(a, b, a_values=None, b_values=None, params: Params | None = None, out=
     _require_cuda(out, "out")
     if out.numel() != a.numel() + b.numel():
         raise ValueError("out must hold a.numel() + b.numel() keys")
-    if a_values is not None and out_values is None:
-        out_values = torch.empty_like(out)
+    if b.device != a.device:
+        raise BcfError("a and b are on different devices")
+    _require_out(out, "out", a.numel() + b.numel(), a.device)
+    if a_values is not None:
+        _require_out(a_values, "a_values", a.numel(), a.device)
+        _require_out(b_values, "b_values", b.numel(), a.device)
+        if out_values is None:
+            out_values = torch.empty_like(out)
+        _require_out(out_values, "out_values", out.numel(), a.device)
     L = lib()
     tb = ctypes.c_size_t(0)
     pp = ctypes.byref(params) if params is not None else None

@@ -488,7 +488,9 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   const uint64_t n = nruns > 0 ? h_run_offsets[nruns] : 0;
   for (int r = 0; r < nruns; ++r)
     if (h_run_offsets[r + 1] < h_run_offsets[r] || h_run_offsets[0] != 0) return BCF_ERROR_INVALID_VALUE;
-  const size_t buf_words = (size_t)n + 4 * ((size_t)nruns + 2) + 64;
+  // per output run: up to 3 phase words + 4 words of gap; per reversed B run
+  // before pass 1: up to 3 phase words + 8 words of gap
+  const size_t buf_words = (size_t)n + 12 * ((size_t)nruns + 2) + 64;
   const size_t key_bytes = align_up(buf_words * sizeof(uint32_t), 256);
   const size_t table_bytes = align_up(sizeof(GroupDesc) * (size_t)(nruns / 2 + 1), 256);
   // + one buffer (per array) for the odd runs reversed before pass 1

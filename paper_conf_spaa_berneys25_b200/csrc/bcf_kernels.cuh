@@ -66,8 +66,9 @@ struct MergeArgs {
   const GroupDesc* groups;  // table mode (merge of arbitrary runs) if non-null
   int ngroups;
   unsigned long long* trace;  // debug timeline (BCF_TRACE), nullptr normally
-  // table mode, plain kernel only: B runs read from these bases instead of
-  // src_k / src_v (bcf_merge_u32: A and B in separate arrays); nullptr = same
+  // table mode (plain and window kernels): B runs read from these bases
+  // instead of src_k / src_v (bcf_merge_u32: A and B in separate arrays;
+  // bcf_merge_runs_u32 pass 1: B runs reversed into temp); nullptr = same
   const uint32_t* src_kb;
   const uint32_t* src_vb;
 };

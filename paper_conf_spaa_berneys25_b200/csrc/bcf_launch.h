@@ -17,7 +17,7 @@ struct Variant {
   MergeFn merge = nullptr;        // regular pass (CF: B runs stored descending)
   MergeFn merge_table = nullptr;  // group-table pass, all runs ascending (CF)
   MergeFn merge_tma = nullptr;    // persistent TMA pass (CF, E coprime with 32); grid arg = tiles
-  MergeFn merge_win = nullptr;    // the persistent window kernel itself (keys only), or nullptr
+  MergeFn merge_win = nullptr;    // the persistent window kernel itself (keys or pairs; reads src_kb/src_vb), or nullptr
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]

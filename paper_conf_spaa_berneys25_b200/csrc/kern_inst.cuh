@@ -2,6 +2,7 @@
 // three block sizes; included by kern_E<E>.cu with BCF_E defined.
 #pragma once
 #include <cstdlib>
+#include <mutex>
 
 #include "bcf_kernels.cuh"
 #include "bcf_merge_tma.cuh"
@@ -74,8 +75,11 @@ cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
 // persistent TMA merge pass: grid = min(tiles, SMs x resident CTAs), each
 // CTA a contiguous, balanced chunk of tiles
 struct PersistentCache {
+  // filled once per device under `mu`; per_sm is published last (release)
+  // and read first (acquire), so a reader that sees it non-zero sees nsm
   int per_sm[32] = {0};
   int nsm[32] = {0};
+  std::mutex mu;
 };
 
 template <typename K>
@@ -85,21 +89,24 @@ cudaError_t launch_persistent(K kern, PersistentCache& pc, size_t smem, int thre
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (dev >= 32) return cudaErrorInvalidDevice;
-  if (pc.per_sm[dev] == 0) {
-    if (smem > 48 * 1024) {
-      e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      if (e != cudaSuccess) {
-        (void)cudaGetLastError();
-        return e;
+  if (__atomic_load_n(&pc.per_sm[dev], __ATOMIC_ACQUIRE) == 0) {
+    std::lock_guard<std::mutex> lk(pc.mu);
+    if (pc.per_sm[dev] == 0) {
+      if (smem > 48 * 1024) {
+        e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) {
+          (void)cudaGetLastError();
+          return e;
+        }
       }
+      int k = 0, sms = 0;
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, threads, smem);
+      if (e != cudaSuccess) return e;
+      e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      if (e != cudaSuccess) return e;
+      pc.nsm[dev] = sms;
+      __atomic_store_n(&pc.per_sm[dev], k > 0 ? k : 1, __ATOMIC_RELEASE);
     }
-    int k = 0, sms = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k, kern, threads, smem);
-    if (e != cudaSuccess) return e;
-    e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (e != cudaSuccess) return e;
-    pc.nsm[dev] = sms;
-    pc.per_sm[dev] = k > 0 ? k : 1;
   }
   // one wave of SMs x resident CTAs, tiles spread evenly (per_cta = 0)
   long long ctas = (long long)pc.nsm[dev] * pc.per_sm[dev];

@@ -165,6 +165,12 @@ def sort(keys, values=None, group=None, ops=None, timing: list | None = None):
     import torch.distributed as dist
 
     ops = ops or CudaOps()
+    if getattr(keys, "dtype", None) is not None and str(keys.dtype) == "torch.float32":
+        # the local sort orders float32 by IEEE totalOrder, but the splitters
+        # and the run merge compare u32 bit patterns: pass keys as int32 bit
+        # patterns (or totalOrder-encoded) instead of relying on a silent mismatch
+        raise TypeError("dist.sort sorts 32-bit keys as unsigned bit patterns: pass int32 (uint32 bits), "
+                        "not float32")
     device = keys.device
     p = dist.get_world_size(group)
     marks = _PhaseMarks(device, timing is not None and p > 1)

@@ -296,6 +296,41 @@ def test_merge_runs_large(sizes, keyspace, params):
     np.testing.assert_array_equal(to_host(vo), ev)
 
 
+@pytest.mark.parametrize("nruns", [54, 62, 64])
+def test_merge_runs_many_runs_with_empty_a_runs(nruns):
+    """with nearly empty A (even) runs, pass 1 places every reversed
+    B run at up to 3 phase words + an 8-word gap; the temp layout must hold
+    ~11 extra words per B run (62 runs, odd runs of 49..79 keys)."""
+    rng = np.random.default_rng(nruns)
+    sizes = [0 if r % 2 == 0 else 49 + (r * 7) % 31 for r in range(nruns)]
+    runs = [np.sort(rng.integers(0, 1 << 32, size=s, dtype=np.uint64).astype(np.uint32)) for s in sizes]
+    keys = np.concatenate(runs)
+    vals = np.arange(keys.size, dtype=np.uint32)
+    offs = np.concatenate([[0], np.cumsum(sizes)]).astype(np.uint64)
+    ek, ev = oracle.sort_pairs_u32(keys, vals)
+    np.testing.assert_array_equal(to_host(bcf.merge_runs(to_dev(keys), offs)), ek)
+    ko, vo = bcf.merge_runs(to_dev(keys), offs, values=to_dev(vals))
+    np.testing.assert_array_equal(to_host(ko), ek)
+    np.testing.assert_array_equal(to_host(vo), ev)
+
+
+def test_wrappers_reject_bad_buffers():
+    """The Python binding checks sizes and devices before any launch."""
+    x = to_dev(si.uniform_u32(1000, 5))
+    with pytest.raises(bcf.BcfError):
+        bcf.sort(x, out=torch.empty(999, dtype=torch.int32, device=DEV))
+    with pytest.raises(bcf.BcfError):
+        bcf.sort_pairs(x, x.clone(), keys_out=torch.empty(10, dtype=torch.int32, device=DEV))
+    with pytest.raises(bcf.BcfError):
+        bcf.merge_runs(x, np.array([0, 500, 1001], dtype=np.uint64))
+    with pytest.raises(bcf.BcfError):
+        bcf.merge_runs(x, np.array([0, 500, 1000], dtype=np.uint64), values=x[:999].clone())
+    with pytest.raises(bcf.BcfError):
+        bcf.merge(x[:500], x[500:], a_values=x[:499].clone(), b_values=x[500:].clone())
+    with pytest.raises(bcf.BcfError):
+        bcf.sort_pairs(x, torch.zeros(1000, dtype=torch.int32))  # values on the CPU
+
+
 MERGE_SIZES = [(0, 0), (0, 5), (7, 0), (1, 1), (3968 * 3 + 17, 5000), (100000, 1), (1, 100000),
                (70001, 70003), (4352, 4352), (1 << 20, (1 << 20) - 3)]
 
