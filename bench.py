@@ -10,12 +10,15 @@ alternate random / worst-case (ABAB) so clock drift cancels in the ratio; L2
 is flushed (256 MiB write) between timed steps, outside the events.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--log2n L]
 
-N > 1 (torchrun, one rank per GPU, NCCL): each rank holds 2^24 keys (weak
-scaling) and a step is the distributed sort (local sort, exact splitters,
-all_to_all, run merge).  Rank 0 prints ONE JSON line.
-`--impl reference` times the CPU oracle (plain stable mergesort, 1 core) on a
-bounded sample of the same workload.
+N > 1 (torchrun, one rank per GPU, NCCL): BASELINE configs[4], 2^32 keys in
+total (2^32 / N per rank, strong scaling), a step is the distributed sort
+(local sort, exact splitters, all_to_all, run merge).  `--gpus 1 --log2n 32`
+runs the same 2^32-key workload on one GPU.  Rank 0 prints ONE JSON line.
+`--impl reference` times the CPU oracle (plain stable mergesort, 1 core) on
+the same workload: the full input per step when the run fits a few minutes,
+else a bounded sample (stated in cpu_baseline.sample).
 """
 from __future__ import annotations
 
@@ -36,7 +39,9 @@ import synthetic_inputs as si  # noqa: E402
 
 METRIC = "sorted keys/s (32-bit) random vs worst-case, ratio; SMEM bank conflicts (ncu)"
 UNIT = "keys/s"
-WORKLOAD = "2^24 uint32 keys, random vs worst-case bank-conflict input, 1xB200 (BASELINE configs[1])"
+WORKLOAD_1 = "2^24 uint32 keys, random vs worst-case bank-conflict input, 1xB200 (BASELINE configs[1])"
+WORKLOAD_DIST = "2^32 uint32 keys distributed sort (splitters + NCCL all-to-all over NVLink) (BASELINE configs[4])"
+REF_BUDGET_S = 150.0  # the reference arm's whole run (warmup + steps) stays within a few minutes
 L2_FLUSH_BYTES = 256 << 20
 DEFAULT_E, DEFAULT_U = 31, 128  # = bcf_default_params()
 
@@ -47,12 +52,47 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--log2n", type=int, default=24)
+    ap.add_argument("--log2n", type=int, default=0, help="total keys 2^L (default 24 at N=1, 32 at N>1)")
     ap.add_argument("--E", type=int, default=0)
     ap.add_argument("--u", type=int, default=0)
     ap.add_argument("--algo", type=int, default=0)
     ap.add_argument("--no-extras", action="store_true", help="skip e2e/cpu_baseline/contrast legs")
     return ap.parse_args()
+
+
+def log2n_total(a, world):
+    return a.log2n or (24 if world == 1 else 32)
+
+
+def workload_config(a, world, E, u):
+    """The `config` object, identical in both arms (ours / reference)."""
+    L = log2n_total(a, world)
+    n = 1 << L
+    if L == 24 and world == 1:
+        wl = WORKLOAD_1
+    elif L == 32:
+        wl = WORKLOAD_DIST if world > 1 else "2^32 uint32 keys, random vs worst-case, 1xB200 (BASELINE configs[4] at N=1)"
+    else:
+        wl = f"2^{L} uint32 keys, random vs worst-case, {world}xB200"
+    return {"workload": wl, "n": n, "n_per_gpu": n // world, "E": E, "u": u,
+            "algo": "conflict_free" if a.algo == 0 else "baseline",
+            "steps_alternate": "random, worst-case (ABAB)",
+            "l2": "flushed between timed steps (256 MiB write, outside the events)",
+            "parallelism": f"dp{world}" if world > 1 else "single"}
+
+
+def cpu_info():
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model,
+            "affinity_cores": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else None}
 
 
 def measured_peaks():
@@ -123,23 +163,32 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def cpu_oracle_rate(n_sample: int, reps: int, kinds, E, u):
-    """The oracle (plain stable mergesort in C, 1 thread) on bounded samples."""
+def cpu_baselines(n: int, E: int, u: int, x_rand: np.ndarray, x_worst: np.ndarray):
+    """(i) the oracle (plain stable mergesort in C, 1
+    thread), (ii) std::stable_sort (1 thread), (iii) a std::thread parallel
+    stable mergesort on all host cores; each on the same random and
+    worst-case inputs as the GPU run (full size), outputs cross-checked."""
     import oracle
-    from oracle import worstcase as wc
 
-    total_keys, total_s = 0, 0.0
-    for i in range(reps):
-        kind = kinds[i % len(kinds)]
-        if kind == "random":
-            x = si.uniform_u32(n_sample, si.config_seed(1) + i)
-        else:
-            x = wc.worst_case_input(n_sample, E, u, si.config_seed(1) + i)
-        t = time.perf_counter()
-        oracle.sort_u32(x)
-        total_s += time.perf_counter() - t
-        total_keys += n_sample
-    return total_keys / total_s, total_s
+    info = cpu_info()
+    cores = info["affinity_cores"] or info["nproc"] or 1
+    res = {}
+    exp = None
+    for name, fn, c in [("oracle", oracle.sort_u32, 1), ("std_stable_sort", oracle.std_stable_sort_u32, 1),
+                        ("parallel_mergesort", lambda x: oracle.parallel_mergesort_u32(x, cores), cores)]:
+        secs = 0.0
+        outs = []
+        for x in (x_rand, x_worst):
+            t = time.perf_counter()
+            outs.append(fn(x))
+            secs += time.perf_counter() - t
+        if exp is None:
+            exp = outs
+        ok = all(np.array_equal(o, e) for o, e in zip(outs, exp))
+        res[name] = {"value": 2 * n / secs, "unit": UNIT, "cores": c, "seconds": secs, "matches_oracle": ok}
+    res["sample"] = f"one random + one worst-case sort of {n} keys each (the full workload)"
+    res.update(info)
+    return res
 
 
 def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
@@ -233,16 +282,24 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
 
 def run_reference(a):
     rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(a.gpus)))
     if rank != 0:
         return 0
     # the library's default (E, u) (tests/test_capi_host.py keeps these equal);
     # the reference arm runs no library code
     E, u = a.E or DEFAULT_E, a.u or DEFAULT_U
-    n_full = 1 << a.log2n
-    n_sample = min(n_full, 1 << 21)
+    n_full = 1 << log2n_total(a, world)
     import oracle
     from oracle import worstcase as wc
 
+    # sample size: the full workload unless warmup + steps would exceed the
+    # budget at the oracle's measured rate (~1 core, n log n)
+    probe = si.uniform_u32(1 << 20, si.config_seed(1))
+    t = time.perf_counter()
+    oracle.sort_u32(probe)
+    per_key = (time.perf_counter() - t) / (1 << 20) * (np.log2(n_full) / 20.0)
+    budget_keys = int(REF_BUDGET_S / max(1, a.steps + a.warmup) / per_key)
+    n_sample = n_full if budget_keys >= n_full else max(1 << 16, budget_keys)
     inputs = [si.uniform_u32(n_sample, si.config_seed(1)), wc.worst_case_input(n_sample, E, u, si.config_seed(1))]
     for i in range(a.warmup):
         oracle.sort_u32(inputs[i % 2])
@@ -255,25 +312,54 @@ def run_reference(a):
     value = a.steps * n_sample / total
     rnd = [t for i, t in enumerate(times) if i % 2 == 0]
     wst = [t for i, t in enumerate(times) if i % 2 == 1]
-    sample = f"{n_sample} keys per step (2^{n_sample.bit_length() - 1} of the 2^{a.log2n} workload), random/worst alternating"
+    if n_sample == n_full:
+        sample = f"the full workload: {n_sample} keys per step, random / worst-case alternating"
+    else:
+        sample = (f"{n_sample} keys per step (of the {n_full}-key workload, bounded to ~{REF_BUDGET_S:.0f} s), "
+                  "random / worst-case alternating")
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": a.gpus,
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * total / a.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
-        "data": "synthetic", "config": {"workload": WORKLOAD, "n": n_full, "E": E, "u": u},
+        "higher_is_better": True, "scaling": "weak" if world == 1 else "strong", "vs_baseline": None,
+        "dtype": "u32", "data": "synthetic", "config": workload_config(a, world, E, u),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                         **cpu_info()},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "random_keys_per_s": len(rnd) * n_sample / sum(rnd) if rnd else None,
         "worst_keys_per_s": len(wst) * n_sample / sum(wst) if wst else None,
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
-        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "worst_over_random_time": (statistics.mean(wst) / statistics.mean(rnd)) if rnd and wst else None,
     }
     print(json.dumps(line))
     return 0
+
+
+def gen_uniform(n, seed, dev, lo=0, chunk=1 << 27):
+    """Rank's shard [lo, lo + n) of the global uniform u32 stream, generated on
+    the device in chunks (bounded temporaries at 2^32 keys)."""
+    import torch
+
+    t = torch.empty(n, dtype=torch.int32, device=dev)
+    for c in range(0, n, chunk):
+        m = min(chunk, n - c)
+        t[c:c + m] = si.uniform_u32_torch(m, seed, dev, lo=lo + c)
+    return t
+
+
+def host_mem_available():
+    try:
+        import psutil
+
+        return psutil.virtual_memory().available
+    except Exception:  # noqa: BLE001
+        return 0
 
 
 def main():
     a = parse()
     if a.impl == "reference":
         return run_reference(a)
+    import ctypes
+
     import torch
     import torch.distributed as dist
 
@@ -293,34 +379,33 @@ def main():
     E = a.E or dp.items_per_thread
     u = a.u or dp.block_threads
     params = bcf.make_params(E, u, a.algo)
-    n = 1 << a.log2n
+    L = log2n_total(a, world)
+    n_total = 1 << L
+    lo = (rank * n_total) // world
+    n = ((rank + 1) * n_total) // world - lo
     seed = si.config_seed(1)
+    config = workload_config(a, world, E, u)
 
     # inputs resident in HBM: rank r's shard of the global random stream, and
-    # the constructed worst case for (E, u)
-    x_rand = si.uniform_u32_torch(n, seed, dev, lo=rank * n)
+    # the Section-4 worst case for (E, u) built on the device
+    x_rand = gen_uniform(n, seed, dev, lo=lo)
     x_worst = bcf.worst_case(n, E, u, seed + rank, device=dev)
     inputs = [x_rand, x_worst]
     out = torch.empty(n, dtype=torch.int32, device=dev)
-    tq = bcf.sort(x_rand[:1], params=params)  # warm the library
-    del tq
-    import ctypes
-
-    tb = ctypes.c_size_t(0)
-    bcf.lib().bcf_sort_u32(None, None, n, None, ctypes.byref(tb), ctypes.byref(params), None)
-    temp = torch.empty(tb.value, dtype=torch.uint8, device=dev)
+    temp = bcf.temp_buffer(n, params, device=dev)
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+    torch.cuda.synchronize()
 
     dist_marks, dist_sends = [], []
 
-    def step(i, timing=None):
-        x = inputs[i % 2]
+    def step(i, timing=None, x=None):
+        x = inputs[i % 2] if x is None else x
         if world == 1:
-            bcf.sort(x, out=out, params=params, temp=temp)
-        else:
-            _, _, st = bdist.sort(x, ops=bdist.CudaOps(params), timing=timing)
-            if timing is not None:
-                dist_sends.append(st.send_counts)
+            return bcf.sort(x, out=out, params=params, temp=temp)
+        ko, _, st = bdist.sort(x, ops=bdist.CudaOps(params), timing=timing)
+        if timing is not None:
+            dist_sends.append(st.send_counts)
+        return ko
 
     for i in range(max(3, a.warmup)):
         step(i)
@@ -346,7 +431,7 @@ def main():
     # between kernels, so they are taken in a second, identical pass over the
     # same workload right after the headline region (which has none).
     bcf.profile_enable(True)
-    for i in range(min(a.steps, 50)):
+    for i in range(min(a.steps, 50 if L <= 28 else 6)):
         flush.fill_(i)
         step(i, timing=dist_marks if world > 1 else None)
     torch.cuda.synchronize()
@@ -375,15 +460,17 @@ def main():
             "splitters": "exact, 64-ary bisection of the key space + rank-ordered tie split",
         }
     prof_ms = sum(v["total_ms"] for v in prof.values())
-    ms = [s.elapsed_time(e) for s, e in ev]
-    total_ms = sum(ms)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    ms = [s_.elapsed_time(e_) for s_, e_ in ev]
+    # max over ranks of the timed region and of each half (random / worst)
+    rnd_ms = sum(m for i, m in enumerate(ms) if i % 2 == 0)
+    wst_ms = sum(m for i, m in enumerate(ms) if i % 2 == 1)
+    t = torch.tensor([sum(ms), rnd_ms, wst_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms_max = float(t.item())
-    value = a.steps * n * world / (total_ms_max / 1e3)
-    rnd = [m for i, m in enumerate(ms) if i % 2 == 0]
-    wst = [m for i, m in enumerate(ms) if i % 2 == 1]
+    total_ms_max, rnd_ms, wst_ms = (float(v) for v in t.tolist())
+    value = a.steps * n_total / (total_ms_max / 1e3)
+    n_rnd = (a.steps + 1) // 2
+    n_wst = a.steps // 2
 
     peaks, peak_src = measured_peaks()
     plan = bcf.sort_plan(n, params)
@@ -404,16 +491,16 @@ def main():
                 traffic = tr.get("dram_bytes_per_launch")
         bs = prof.get("block_sort")
         in_region = None
-        if bs and bs["launches"] and passes:
+        if bs and bs["launches"] and passes and world == 1:
             # the profiled pass brackets every launch with events, which
             # serialises the launches (no PDL overlap); the headline region has
             # none: its per-pass time, net of the event-timed block sort
             in_region = (total_ms_max / a.steps - bs["total_ms"] / bs["launches"]) / passes
         roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "merge_pass_in_region_est_ms": in_region,
-                "achieved_in_region_est": (bytes_per_launch / (in_region / 1e3) / 1e9) if in_region else None,
                 "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
                 "kernel": "merge_pass", "avg_launch_ms": avg_ms, "bytes_per_launch": bytes_per_launch,
+                "merge_pass_in_region_est_ms": in_region,
+                "achieved_in_region_est": (bytes_per_launch / (in_region / 1e3) / 1e9) if in_region else None,
                 "peak_source": f"hbm_gbs {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}
     kernels = {k: {"launches": v["launches"], "avg_ms": v["total_ms"] / max(1, v["launches"]),
                    "share_of_kernel_time": v["total_ms"] / prof_ms if prof_ms else None}
@@ -422,15 +509,9 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
         "warmup": max(3, a.warmup), "ms_per_step": total_ms_max / a.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": WORKLOAD, "n": n, "n_per_gpu": n, "E": E, "u": u, "tile": T, "block_sort_tile": plan["block_sort_tile"],
-                   "merge_passes": passes, "algo": "conflict_free" if a.algo == 0 else "baseline",
-                   "steps_alternate": "random, worst-case (ABAB)",
-                   "l2": "flushed between timed steps (256 MiB write, outside the events)",
-                   "parallelism": f"dp{world}" if world > 1 else "single"},
-        "random_keys_per_s": len(rnd) * n * world / (sum(rnd) / 1e3) if rnd else None,
-        "worst_keys_per_s": len(wst) * n * world / (sum(wst) / 1e3) if wst else None,
-        "worst_over_random_time": (statistics.mean(wst) / statistics.mean(rnd)) if rnd and wst else None,
+        "scaling": "weak" if world == 1 else "strong", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic", "config": config,
+        "plan": {"tile": T, "block_sort_tile": plan["block_sort_tile"], "merge_passes": passes},
         "roofline": roof,
         "kernels": kernels,
         "gpu_launches": launches,
@@ -439,54 +520,102 @@ def main():
     if distributed is not None:
         line["distributed"] = distributed
 
-    if rank == 0 and world == 1 and not a.no_extras:
-        # e2e through the public C-ABI host-buffer entry point
-        # (bcf_sort_u32_host_batch): every step = H2D of that step's input from
-        # pinned host memory, the sort, D2H of the sorted result; the copies of
-        # neighbouring steps overlap the sort (both copy directions at once).
-        # Inputs alternate random / worst-case as in the headline.
-        hx = [x.cpu().pin_memory() for x in inputs]
+    # ---- e2e through the public API, host buffers, copies inside the region
+    big = n > (1 << 28)
+    if not a.no_extras or world > 1 or big:
+        need = 4 * 4 * n if (world == 1 and not big) else 2 * 4 * n
+        if host_mem_available() > 2 * need * (world if world > 1 else 1):
+            line["e2e"] = e2e_leg(a, bcf, bdist, torch, dist, dev, stream, inputs, out, temp, params, n,
+                                  n_total, world, big)
+        else:
+            line["e2e"] = {"value": None, "unit": UNIT, "skipped": "not enough host memory for pinned buffers",
+                           "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 4 * n}
+
+    if rank == 0 and world == 1 and not a.no_extras and not big:
+        line["contrast"] = contrast_leg(bcf, torch, dev, stream, flush, x_rand, out, n, u, seed, a.steps)
+        line["configs_extra"] = extra_configs(bcf, dev, stream, flush, params, peaks)
+        xr = x_rand.cpu().numpy().view(np.uint32)
+        xw = x_worst.cpu().numpy().view(np.uint32)
+        cb = cpu_baselines(n, E, u, xr, xw)
+        orc = cb.pop("oracle")
+        line["cpu_baseline"] = {"value": orc["value"], "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": cb.pop("sample"), **cb}
+    # the headline ratio last, so it survives any tail truncation of stdout
+    line["random_keys_per_s"] = n_rnd * n_total / (rnd_ms / 1e3) if n_rnd else None
+    line["worst_keys_per_s"] = n_wst * n_total / (wst_ms / 1e3) if n_wst else None
+    line["worst_over_random_time"] = ((wst_ms / n_wst) / (rnd_ms / n_rnd)) if n_rnd and n_wst else None
+    if rank == 0:
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def e2e_leg(a, bcf, bdist, torch, dist, dev, stream, inputs, out, temp, params, n, n_total, world, big):
+    """The metric end to end through the public API: every step copies that
+    step's input from pinned host memory to the device, sorts it, and reads
+    the sorted keys back; the copies are inside the timed region."""
+    hx = [x.cpu().pin_memory() for x in inputs]
+    if world == 1 and not big:
+        # bcf_sort_u32_host_batch: H2D / sort / D2H of consecutive steps overlap
         hy = [torch.empty(n, dtype=torch.int32).pin_memory() for _ in range(2)]
         ke = min(a.steps, 40)
         h_in = [hx[i % 2] for i in range(ke)]
         h_out = [hy[i % 2] for i in range(ke)]
-        htemp = None
         bcf.sort_host_batch(h_in[:4], h_out[:4], params=params, device=dev)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        bcf.sort_host_batch(h_in, h_out, params=params, temp=htemp, device=dev)
+        bcf.sort_host_batch(h_in, h_out, params=params, device=dev)
         e1.record(stream)
         torch.cuda.synchronize()
-        e2e_ms = e0.elapsed_time(e1)
-        line["e2e"] = {"value": ke * n / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": 4 * n,
-                       "d2h_bytes_per_step": 4 * n, "steps": ke,
-                       "api": "bcf_sort_u32_host_batch (pinned host buffers, H2D/sort/D2H of consecutive steps overlap)"}
-        # the same, one step per call (no overlap between steps): context
-        dx = torch.empty(n, dtype=torch.int32, device=dev)
-        e2e_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(10)]
-        for i in range(10):
-            e2e_ev[i][0].record(stream)
-            dx.copy_(hx[i % 2], non_blocking=True)
-            bcf.sort(dx, out=out, params=params, temp=temp)
-            hy[i % 2].copy_(out, non_blocking=True)
-            e2e_ev[i][1].record(stream)
-        torch.cuda.synchronize()
-        ser_ms = sum(s_.elapsed_time(e_) for s_, e_ in e2e_ev)
-        line["e2e_one_step_per_call"] = {"value": 10 * n / (ser_ms / 1e3), "unit": UNIT}
+        return {"value": ke * n / (e0.elapsed_time(e1) / 1e3), "unit": UNIT, "h2d_bytes_per_step": 4 * n,
+                "d2h_bytes_per_step": 4 * n, "steps": ke,
+                "api": "bcf_sort_u32_host_batch (pinned host buffers, H2D/sort/D2H of consecutive steps overlap)"}
+    # one step per call: H2D, sort (distributed at N > 1), D2H; max over ranks
+    hy = torch.empty(n, dtype=torch.int32).pin_memory()
+    dx = torch.empty(n, dtype=torch.int32, device=dev)
+    ke = 4
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(ke)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(ke):
+        evs[i][0].record(stream)
+        dx.copy_(hx[i % 2], non_blocking=True)
+        if world == 1:
+            r = bcf.sort(dx, out=out, params=params, temp=temp)
+        else:
+            r, _, _ = bdist.sort(dx, ops=bdist.CudaOps(params))
+        hr = hy[:r.numel()]
+        hr.copy_(r, non_blocking=True)
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    tot = torch.tensor([sum(s_.elapsed_time(e_) for s_, e_ in evs)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    return {"value": ke * n_total / (float(tot.item()) / 1e3), "unit": UNIT, "h2d_bytes_per_step": 4 * n,
+            "d2h_bytes_per_step": 4 * n, "steps": ke,
+            "api": ("dist.sort (one step per call: H2D of the rank's shard, distributed sort, D2H of the "
+                    "rank's output), max over ranks") if world > 1 else
+                   "bcf.sort (one step per call: H2D, sort, D2H; no overlap)"}
 
-        # contrast: the unmodified-Thrust baseline variant on the same inputs
-        bp = bcf.make_params(E if E in (15, 17) else 15, u, bcf.ALGO_BASELINE)
-        contrast = {}
-        for name, prm in [("baseline_thrust", bp), ("cf_same_E", bcf.make_params(bp.items_per_thread, u, 0))]:
-            xw = bcf.worst_case(n, prm.items_per_thread, u, seed, device=dev)
+
+def contrast_leg(bcf, torch, dev, stream, flush, x_rand, out, n, u, seed, steps):
+    """The unmodified-Thrust baseline variant (BCF_ALGO_BASELINE) on the same
+    random input and on the Section-4 worst case built for ITS (E, u), beside
+    the CF kernels with the same (E, u): E = 31 (our default) and E = 15 (the
+    paper's, P:356)."""
+    contrast = {}
+    for E_ in (31, 15):
+        for name, algo in (("baseline_thrust", bcf.ALGO_BASELINE), ("cf", 0)):
+            prm = bcf.make_params(E_, u, algo)
+            xw = bcf.worst_case(n, E_, u, seed, device=dev)
             ins = [x_rand, xw]
-            tbb = ctypes.c_size_t(0)
-            bcf.lib().bcf_sort_u32(None, None, n, None, ctypes.byref(tbb), ctypes.byref(prm), None)
-            tmp2 = torch.empty(tbb.value, dtype=torch.uint8, device=dev)
+            tmp2 = bcf.temp_buffer(n, prm, device=dev)
             for i in range(4):
                 bcf.sort(ins[i % 2], out=out, params=prm, temp=tmp2)
-            kc = min(a.steps, 60)
+            kc = min(steps, 60)
             cev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(kc)]
             for i in range(kc):
                 flush.fill_(i)
@@ -497,22 +626,12 @@ def main():
             cm = [s.elapsed_time(e) for s, e in cev]
             r_ = [m for i, m in enumerate(cm) if i % 2 == 0]
             w_ = [m for i, m in enumerate(cm) if i % 2 == 1]
-            contrast[name] = {"E": prm.items_per_thread, "u": u,
-                              "random_keys_per_s": len(r_) * n / (sum(r_) / 1e3),
-                              "worst_keys_per_s": len(w_) * n / (sum(w_) / 1e3),
-                              "worst_over_random_time": statistics.mean(w_) / statistics.mean(r_)}
-        line["contrast"] = contrast
-
-        line["configs_extra"] = extra_configs(bcf, dev, stream, flush, params, peaks)
-
-        rate, secs = cpu_oracle_rate(n, 3, ["random", "worst", "random"], E, u)
-        line["cpu_baseline"] = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-                                "sample": f"3 sorts of {n} keys (random, worst-case, random), {secs:.1f} s on 1 core"}
-    if rank == 0:
-        print(json.dumps(line))
-    if world > 1:
-        dist.destroy_process_group()
-    return 0
+            contrast[f"{name}_E{E_}"] = {"E": E_, "u": u,
+                                         "random_keys_per_s": len(r_) * n / (sum(r_) / 1e3),
+                                         "worst_keys_per_s": len(w_) * n / (sum(w_) / 1e3),
+                                         "worst_over_random_time": statistics.mean(w_) / statistics.mean(r_)}
+            del xw, tmp2
+    return contrast
 
 
 if __name__ == "__main__":

@@ -8,6 +8,9 @@ paper_conf_spaa_berneys25_b200 computes, written from the paper
     addrmap.py      pi, rho and Alg. 1's gather schedule (§3)
     dmm.py          DMM bank-conflict cost model + Thrust serial-merge address stream
     worstcase.py    Section 4 worst-case construction (S, T, Theorem 8) + composition
+    cpu_baselines.cpp  std::stable_sort (1 core) and a std::thread parallel
+                    stable mergesort (all cores): the further CPU baselines of
+                    SURVEY.md §8(d), also a library cross-check of the oracle
 
 Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
 `--impl reference` leg may import, call, link or execute anything under
@@ -33,13 +36,53 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
+_CPP_SRC = os.path.join(_HERE, "cpu_baselines.cpp")
+_CPP_LIB = os.path.join(_HERE, "libcpu_baselines.so")
+_cpp = None
+
+
 def build(force: bool = False) -> str:
-    """Compile sort_oracle.c with gcc (plain C, -O2, single thread)."""
+    """Compile sort_oracle.c with gcc (plain C, -O2, single thread) and the
+    CPU baselines with g++ (-O2, std::thread)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         subprocess.check_call(
             ["gcc", "-O2", "-std=c99", "-shared", "-fPIC", "-o", _LIB, _SRC]
         )
+    if force or not os.path.exists(_CPP_LIB) or os.path.getmtime(_CPP_LIB) < os.path.getmtime(_CPP_SRC):
+        subprocess.check_call(
+            ["g++", "-O2", "-std=c++17", "-pthread", "-shared", "-fPIC", "-o", _CPP_LIB, _CPP_SRC]
+        )
     return _LIB
+
+
+def cpp_lib():
+    global _cpp
+    if _cpp is None:
+        build()
+        L = ctypes.CDLL(_CPP_LIB)
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        L.baseline_std_stable_sort_u32.argtypes = [u32p, u32p, ctypes.c_uint64]
+        L.baseline_std_stable_sort_u32.restype = ctypes.c_int
+        L.baseline_parallel_mergesort_u32.argtypes = [u32p, u32p, ctypes.c_uint64, ctypes.c_int]
+        L.baseline_parallel_mergesort_u32.restype = ctypes.c_int
+        _cpp = L
+    return _cpp
+
+
+def std_stable_sort_u32(keys: np.ndarray) -> np.ndarray:
+    """CPU baseline (ii): std::stable_sort on one core."""
+    k = np.ascontiguousarray(keys, dtype=np.uint32)
+    out = np.empty_like(k)
+    cpp_lib().baseline_std_stable_sort_u32(_p(k), _p(out), k.size)
+    return out
+
+
+def parallel_mergesort_u32(keys: np.ndarray, threads: int) -> np.ndarray:
+    """CPU baseline (iii): chunked std::stable_sort + parallel std::merge tree."""
+    k = np.ascontiguousarray(keys, dtype=np.uint32)
+    out = np.empty_like(k)
+    cpp_lib().baseline_parallel_mergesort_u32(_p(k), _p(out), k.size, int(threads))
+    return out
 
 
 def lib():

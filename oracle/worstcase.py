@@ -256,8 +256,17 @@ def worst_case_input(n: int, E: int, u: int, seed: int, w: int = 32) -> np.ndarr
             pair_abs = (g0[irr] + pi - (pi & 1)) // 2
             bit = (stream_np(seed_l, pair_abs) >> np.uint64(63)).astype(np.int64)
             label_B[irr] = (pi < 2 * nb) & (((pi & 1) ^ bit) == 1)
-        key = g * 2 + label_B.astype(np.int64)
-        vals = vals[np.argsort(key, kind="stable")]
+        # stable partition of every group: the A-labelled outputs, in order,
+        # fill the A child [g0, g0 + na), the B-labelled ones the B child
+        isA = ~label_B
+        cumA = np.cumsum(isA) - isA                      # A labels before p
+        cumB = np.cumsum(label_B) - label_B              # B labels before p
+        rankA = cumA - cumA[g0]
+        rankB = cumB - cumB[g0]
+        dest = np.where(isA, g0 + rankA, g0 + na + rankB)
+        nxt = np.empty_like(vals)
+        nxt[dest] = vals
+        vals = nxt
     # bottom: shuffle every run of E (one thread's items); Fisher-Yates with
     # j = floor(hi32(h) * (i + 1) / 2^32)
     seed_s = (seed + SHUFFLE_SALT) & MASK64

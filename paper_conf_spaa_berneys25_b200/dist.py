@@ -63,6 +63,50 @@ class DistStats:
     pivots: list | None = None
 
 
+def _staged(group) -> bool:
+    """gloo cannot run collectives on CUDA tensors: stage them through host
+    copies (a correctness path for the world-size-2 test on one GPU; the
+    product's multi-GPU path is NCCL)."""
+    import torch.distributed as dist
+
+    return dist.get_backend(group) == "gloo"
+
+
+def _all_reduce(t, group):
+    import torch.distributed as dist
+
+    if t.is_cuda and _staged(group):
+        h = t.cpu()
+        dist.all_reduce(h, group=group)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, group=group)
+
+
+def _all_gather(outs, t, group):
+    import torch.distributed as dist
+
+    if t.is_cuda and _staged(group):
+        ho = [o.cpu() for o in outs]
+        dist.all_gather(ho, t.cpu(), group=group)
+        for o, h in zip(outs, ho):
+            o.copy_(h)
+    else:
+        dist.all_gather(outs, t, group=group)
+
+
+def _all_to_all(out, inp, group, out_splits=None, in_splits=None):
+    import torch.distributed as dist
+
+    if inp.is_cuda and _staged(group):
+        ho = out.cpu()
+        dist.all_to_all_single(ho, inp.cpu(), output_split_sizes=out_splits, input_split_sizes=in_splits,
+                               group=group)
+        out.copy_(ho)
+    else:
+        dist.all_to_all_single(out, inp, output_split_sizes=out_splits, input_split_sizes=in_splits, group=group)
+
+
 def _targets(N: int, p: int):
     return [(t * N) // p for t in range(1, p)]
 
@@ -76,7 +120,7 @@ def exact_splitters(sorted_keys, n_local: int, group, ops, device):
     p = dist.get_world_size(group)
     r = dist.get_rank(group)
     nt = torch.tensor([n_local], dtype=torch.int64, device=device)
-    dist.all_reduce(nt, group=group)
+    _all_reduce(nt, group)
     N = int(nt.item())
     ks = _targets(N, p)
     lo = [0] * (p - 1)           # answer in [lo, hi]
@@ -96,7 +140,7 @@ def exact_splitters(sorted_keys, n_local: int, group, ops, device):
         piv_np = np.array(piv, dtype=np.uint64).astype(np.uint32)
         _, le = ops.split_counts(sorted_keys, piv_np)
         le = le.to(torch.int64)
-        dist.all_reduce(le, group=group)
+        _all_reduce(le, group)
         le_h = le.cpu().numpy()
         for t in range(p - 1):
             if hi[t] <= lo[t]:
@@ -116,7 +160,7 @@ def exact_splitters(sorted_keys, n_local: int, group, ops, device):
     eq = le.to(torch.int64) - lt
     both = torch.stack([lt, eq])                       # [2, p-1]
     gathered = [torch.empty_like(both) for _ in range(p)]
-    dist.all_gather(gathered, both, group=group)
+    _all_gather(gathered, both, group)
     G = torch.stack(gathered).cpu().numpy()            # [p, 2, p-1]
     cuts = [0]
     for t in range(p - 1):
@@ -182,15 +226,15 @@ def sort(keys, values=None, group=None, ops=None, timing: list | None = None):
     send, pivots, rounds = exact_splitters(sk, sk.numel(), group, ops, device)
     sc = torch.tensor(send, dtype=torch.int64, device=device)
     rc = torch.empty_like(sc)
-    dist.all_to_all_single(rc, sc, group=group)
+    _all_to_all(rc, sc, group)
     recv = [int(x) for x in rc.cpu().tolist()]
     marks.mark()
     rk = torch.empty(sum(recv), dtype=keys.dtype, device=device)
-    dist.all_to_all_single(rk, sk, output_split_sizes=recv, input_split_sizes=send, group=group)
+    _all_to_all(rk, sk, group, recv, send)
     rv = None
     if sv is not None:
         rv = torch.empty(sum(recv), dtype=values.dtype, device=device)
-        dist.all_to_all_single(rv, sv, output_split_sizes=recv, input_split_sizes=send, group=group)
+        _all_to_all(rv, sv, group, recv, send)
     marks.mark()
     offs = np.concatenate([[0], np.cumsum(recv)]).astype(np.uint64)
     ok, ov = ops.merge_runs(rk, offs, rv)

@@ -399,24 +399,82 @@ def test_full_2p26_pairs():
     np.testing.assert_array_equal(to_host(vo), ev)
 
 
-def test_full_2p28_f32_properties():
-    """2^28 f32: sampled oracle check is impractical element by element, so
-    check properties that hold at any size: output non-decreasing in
-    totalOrder and a permutation of the input (equal to torch's sort of the
-    input as a multiset), plus an exact oracle check on a 2^22 prefix-sort."""
+def test_full_2p28_f32_against_oracle():
+    """BASELINE configs[2]: 2^28 f32 in the bench configuration, compared with
+    the oracle (totalOrder mergesort, 1 core, ~40 s) element by element."""
     n = 1 << 28
     x = si.uniform_f32(n, si.config_seed(6))
-    t = torch.from_numpy(x).to(DEV)
+    out = bcf.sort(torch.from_numpy(x).to(DEV))
+    torch.cuda.synchronize()
+    got = out.cpu().numpy().view(np.uint32)
+    del out
+    torch.cuda.empty_cache()
+    np.testing.assert_array_equal(got, oracle.sort_f32_bits(x.view(np.uint32)))
+
+
+def _chunked_device_u32(n, seed, chunk=1 << 27):
+    t = torch.empty(n, dtype=torch.int32, device=DEV)
+    for lo in range(0, n, chunk):
+        hi = min(n, lo + chunk)
+        t[lo:hi] = si.uniform_u32_torch(hi - lo, seed, DEV, lo=lo)
+    return t
+
+
+def _check_big_sort_against_oracle(x: np.ndarray, got: np.ndarray, nranges=6, width=1 << 21):
+    """Exact oracle checks for a sort too large to replay whole on one core:
+    (1) the output is non-decreasing and has the input's multiset of keys
+    (per-16-bit-bucket counts); (2) for several key ranges [lo, hi) the output
+    slice at positions [#(x < lo), #(x < hi)) equals the oracle's sort of the
+    input keys in [lo, hi) -- element by element, including the slices at the
+    very start and end of the output (the 64-bit tile offsets past 2^31)."""
+    n = x.size
+    step = 1 << 26
+    for lo in range(0, n - 1, step):
+        hi = min(n, lo + step + 1)
+        assert np.all(got[lo + 1:hi] >= got[lo:hi - 1]), f"not sorted near {lo}"
+    hx = np.zeros(1 << 16, np.int64)
+    hg = np.zeros(1 << 16, np.int64)
+    for lo in range(0, n, step):
+        hx += np.bincount(x[lo:lo + step] >> 16, minlength=1 << 16)
+        hg += np.bincount(got[lo:lo + step] >> 16, minlength=1 << 16)
+    np.testing.assert_array_equal(hx, hg)
+    kmax = int(got[-1])
+    bounds = [0] + [int(v) for v in np.linspace(0, kmax, nranges)[1:-1]] + [max(0, kmax - width * 4)]
+    for klo in bounds:
+        khi = min(klo + width * 4, 1 << 32)
+        sel = np.concatenate([x[lo:lo + step][(x[lo:lo + step] >= klo) & (x[lo:lo + step] < khi)]
+                              for lo in range(0, n, step)])
+        before = int(sum(np.count_nonzero(x[lo:lo + step] < klo) for lo in range(0, n, step)))
+        exp = oracle.sort_u32(sel)
+        np.testing.assert_array_equal(got[before:before + exp.size], exp, err_msg=f"key range [{klo}, {khi})")
+
+
+def test_sort_past_2p31_keys():
+    """n = 2^31 + 12345 (bcf.h promises n up to 2^32): the 64-bit tile offsets
+    and per-pass group arithmetic past 2^31, uniform random keys and the
+    Section-4 worst case (a permutation of 0..n-1, whose sorted order is
+    0..n-1), checked against the oracle as in _check_big_sort_against_oracle."""
+    n = (1 << 31) + 12345
+    t = _chunked_device_u32(n, si.config_seed(7))
     out = bcf.sort(t)
     torch.cuda.synchronize()
-    assert bool((out[1:] >= out[:-1]).all())
-    ref, _ = torch.sort(t)
-    assert torch.equal(out, ref)
-    del ref, out, t
-    m = 1 << 22
-    np.testing.assert_array_equal(
-        bcf.sort(torch.from_numpy(x[:m]).to(DEV)).cpu().numpy().view(np.uint32),
-        oracle.sort_f32_bits(x[:m].view(np.uint32)))
+    x = t.cpu().numpy().view(np.uint32)
+    del t
+    got = out.cpu().numpy().view(np.uint32)
+    del out
+    torch.cuda.empty_cache()
+    _check_big_sort_against_oracle(x, got)
+    del x, got
+    w = bcf.worst_case(n, 31, 128, seed=si.config_seed(7))
+    out = bcf.sort(w)
+    torch.cuda.synchronize()
+    del w
+    ok = torch.equal(out, torch.arange(n, dtype=torch.int64, device=DEV).to(torch.int32))
+    got_head = out[:1 << 20].cpu().numpy().view(np.uint32)
+    del out
+    torch.cuda.empty_cache()
+    assert ok
+    np.testing.assert_array_equal(got_head, np.arange(1 << 20, dtype=np.uint32))
 
 
 @pytest.mark.parametrize("nbatch,n", [(1, 1), (3, 4097), (5, 100003), (4, 1 << 20)])

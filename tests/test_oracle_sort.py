@@ -134,3 +134,14 @@ def test_f32_random_bit_patterns_against_key_sort():
 
     exp = sorted((int(b) for b in bits), key=key)
     assert list(oracle.sort_f32_bits(bits)) == exp
+
+
+@pytest.mark.parametrize("n", [0, 1, 7, 1000, 100003, 1 << 20])
+def test_oracle_matches_cpu_baselines(n):
+    """The oracle against the library routine std::stable_sort and the
+    parallel mergesort baseline."""
+    x = si.uniform_u32(n, 99 + n) & np.uint32(0xFFFF if n % 2 else 0xFFFFFFFF)
+    exp = oracle.sort_u32(x)
+    np.testing.assert_array_equal(oracle.std_stable_sort_u32(x), exp)
+    for th in (1, 3, 8):
+        np.testing.assert_array_equal(oracle.parallel_mergesort_u32(x, th), exp)
