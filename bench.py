@@ -257,10 +257,13 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         torch.cuda.synchronize()
         bcf.profile_enable(False)
         prof = bcf.profile_collect()
-        cls = "merge_runs" if name.startswith("merge_runs") else ("merge" if name.startswith("merge") else "merge_pass")
-        mp = prof.get(cls, {"launches": 0, "total_ms": 0.0})
+        cls = "merge_runs" if name.startswith("merge_runs") else ("merge" if name.startswith("merge") else
+                                                                   ("merge_passes" if "merge_passes" in prof
+                                                                    else "merge_pass"))
+        mp = prof.get(cls, {"launches": 0, "total_ms": 0.0, "keys": 0})
         bs = prof.get("block_sort", {"launches": 0, "total_ms": 0.0})
         avg = mp["total_ms"] / max(1, mp["launches"])
+        bpl = bpk * mp["keys"] / max(1, mp["launches"])  # keys counts n per pass
         res[name] = {"workload": workload, "n": n, "E": prm.items_per_thread, "u": prm.block_threads,
                      "value": n / (ms / 1e3),
                      "unit": "pairs/s" if name.startswith("pairs") else "keys/s", "ms_per_sort": ms,
@@ -269,9 +272,9 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
                                     "frac_of_hbm": (8 * n / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
                                     "bytes_per_launch": 8 * n} if name.startswith("merge_runs") else
                                    {"launches_per_sort": mp["launches"] // 3, "avg_ms": avg,
-                                    "achieved_gbs": bpk * n / (avg / 1e3) / 1e9 if avg else None,
-                                    "frac_of_hbm": (bpk * n / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
-                                    "bytes_per_launch": bpk * n},
+                                    "achieved_gbs": bpl / (avg / 1e3) / 1e9 if avg else None,
+                                    "frac_of_hbm": (bpl / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
+                                    "bytes_per_launch": bpl, "passes_per_launch": bpl / (bpk * n)},
                      # merge legs: algorithmic bytes of the whole call / call time
                      "call_gbs_algorithmic": bpk * n / (ms / 1e3) / 1e9 if name.startswith("merge") else None,
                      "block_sort_ms": bs["total_ms"] / max(1, bs["launches"])}
@@ -477,10 +480,13 @@ def main():
     T = plan["merge_tile"]
     passes = plan["merge_passes"]
     roof = None
-    mp = prof.get("merge_pass")
+    mcls = "merge_passes" if "merge_passes" in prof else "merge_pass"
+    mp = prof.get(mcls)
     if mp and mp["launches"]:
         avg_ms = mp["total_ms"] / mp["launches"]
-        bytes_per_launch = 8 * n  # read 4 B + write 4 B per key per pass
+        # read 4 B + write 4 B per key per pass; "keys" counts n per pass
+        # (a merge_passes launch runs every pass of one sort)
+        bytes_per_launch = 8 * mp["keys"] / mp["launches"]
         achieved = bytes_per_launch / (avg_ms / 1e3) / 1e9
         traffic = None
         tf = os.path.join(ROOT, "profiles", "merge_pass_traffic.json")
@@ -494,11 +500,13 @@ def main():
         if bs and bs["launches"] and passes and world == 1:
             # the profiled pass brackets every launch with events, which
             # serialises the launches (no PDL overlap); the headline region has
-            # none: its per-pass time, net of the event-timed block sort
-            in_region = (total_ms_max / a.steps - bs["total_ms"] / bs["launches"]) / passes
+            # none: its merge time per launch, net of the event-timed block sort
+            in_region = (total_ms_max / a.steps - bs["total_ms"] / bs["launches"]) / (
+                passes if mcls == "merge_pass" else 1)
         roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
-                "kernel": "merge_pass", "avg_launch_ms": avg_ms, "bytes_per_launch": bytes_per_launch,
+                "kernel": mcls, "avg_launch_ms": avg_ms, "bytes_per_launch": bytes_per_launch,
+                "passes_per_launch": passes if mcls == "merge_passes" else 1,
                 "merge_pass_in_region_est_ms": in_region,
                 "achieved_in_region_est": (bytes_per_launch / (in_region / 1e3) / 1e9) if in_region else None,
                 "peak_source": f"hbm_gbs {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}

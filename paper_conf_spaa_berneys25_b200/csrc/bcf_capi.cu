@@ -143,18 +143,33 @@ static int bs_threads(const Params& p, bool cf, bool pairs) {
 // BCF_TRACE=<pass>: record a per-CTA timeline of that merge pass (debug)
 static unsigned long long* g_trace = nullptr;
 static const size_t TRACE_WORDS = 1 << 21;
-static unsigned long long* trace_for_pass(int pass) {
+static int trace_pass_wanted() {
   static const int want = [] {
     const char* v = getenv("BCF_TRACE");
     return v ? atoi(v) : -1;
   }();
-  if (pass != want) return nullptr;
+  return want;
+}
+static bool trace_requested() { return trace_pass_wanted() >= 0; }
+static unsigned long long* trace_for_pass(int pass) {
+  if (pass != trace_pass_wanted()) return nullptr;
   if (!g_trace) {
     if (cudaMalloc(&g_trace, TRACE_WORDS * 8) != cudaSuccess) return nullptr;
     cudaMemset(g_trace, 0, TRACE_WORDS * 8);
   }
   return g_trace;
 }
+
+// BCF_NO_MULTI=1: one launch per merge pass instead of every pass of a sort in
+// one persistent launch (A/B measurements)
+static bool multipass_disabled() {
+  static const bool off = [] {
+    const char* v = getenv("BCF_NO_MULTI");
+    return v && v[0] == '1';
+  }();
+  return off;
+}
+static constexpr int MAX_PROGRESS_CTAS = 2048;
 
 // BCF_NO_TMA=1 selects the non-persistent merge kernel (A/B measurements)
 static bool tma_disabled() {
@@ -183,7 +198,8 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   // two ping-pong buffers X, Y (256-B aligned, 64 words of slack for the
   // sigma-shifted descending runs); only the final pass writes d_out
   const size_t key_bytes = align_up(((size_t)n + 64) * sizeof(uint32_t), 256);
-  const size_t need = 256 + key_bytes * 2 * (pairs ? 2 : 1);
+  // + per-CTA progress flags of the multi-pass merge launch
+  const size_t need = 256 + key_bytes * 2 * (pairs ? 2 : 1) + MAX_PROGRESS_CTAS * sizeof(unsigned);
   if (d_temp == nullptr) {
     *temp_bytes = need;
     return BCF_SUCCESS;
@@ -218,10 +234,31 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   uint32_t* XV = pairs ? (uint32_t*)(tb + 2 * key_bytes) : nullptr;
   uint32_t* YV = pairs ? (uint32_t*)(tb + 3 * key_bytes) : nullptr;
 
+  unsigned* progress = (unsigned*)(tb + key_bytes * 2 * (pairs ? 2 : 1));
+
+  // every merge pass in one persistent launch (the window kernel; per-CTA
+  // progress flags instead of pass boundaries), unless a pass needs another
+  // kernel: pairs whose final key / value outputs differ in 16-byte phase
+  // take the plain kernel for the last pass
+  const bool last_phase_ok = !pairs || (((uintptr_t)out_k ^ (uintptr_t)out_v) & 15) == 0;
+  const bool multi = P >= 2 && use_tma && var.merge_multi && last_phase_ok && !multipass_disabled() &&
+                     !trace_requested();
+  // the block sort zeroes the progress flags (no memset between the two launches)
   SortArgs sa{in_k, in_v, P == 0 ? out_k : X, P == 0 ? out_v : XV, (long long)n, f32 ? 1 : 0,
-              (f32 && P == 0) ? 1 : 0, cf ? 1 : 0};
+              (f32 && P == 0) ? 1 : 0, cf ? 1 : 0, multi ? progress : nullptr, multi ? MAX_PROGRESS_CTAS : 0};
   cudaError_t e = launch("block_sort", n, s, [&] { return vbs.block_sort(sa, tiles_bs, s); });
   if (e != cudaSuccess) return cuda_fail(e);
+  if (multi) {
+    MergeArgs ma{X, XV, out_k, out_v, (long long)n, Tbs, 1 + lg_bs, f32 ? 1 : 0, cf ? 1 : 0, nullptr, 0, nullptr};
+    ma.npass = P;
+    ma.progress = progress;
+    ma.buf_k[0] = X;
+    ma.buf_k[1] = Y;
+    ma.buf_v[0] = XV;
+    ma.buf_v[1] = YV;
+    e = launch("merge_passes", n * (uint64_t)P, s, [&] { return var.merge_multi(ma, tiles, s); });
+    return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+  }
   for (int i = 1; i <= P; ++i) {
     uint32_t* sk = (i & 1) ? X : Y;
     uint32_t* sv = (i & 1) ? XV : YV;

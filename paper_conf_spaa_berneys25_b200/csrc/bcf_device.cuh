@@ -90,12 +90,21 @@ __device__ __forceinline__ int rho_partition_end(int k) {
 // descending, so that the tile stage writes B reversed = pi(B) with unit-stride
 // reads).
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
 struct RunView {
   const uint32_t* base;
   long long len;
-  int desc;  // 1: element y lives at base[len-1-y]
+  int desc;      // 1: element y lives at base[len-1-y]
+  int coherent = 0;  // 1: L2-coherent loads (data written earlier in the same launch by other CTAs)
   __device__ __forceinline__ long long addr(long long y) const { return desc ? (len - 1 - y) : y; }
-  __device__ __forceinline__ uint32_t ld(long long y) const { return __ldg(base + addr(y)); }
+  __device__ __forceinline__ uint32_t ld(long long y) const {
+    return coherent ? ld_cg(base + addr(y)) : __ldg(base + addr(y));
+  }
 };
 
 // ---------------------------------------------------------------------------

@@ -44,6 +44,8 @@ struct SortArgs {
   int encode_f32;  // encode f32 -> totalOrder u32 on load (block sort)
   int decode_f32;  // decode on the final store
   int cf_dirs;     // CF run directions (odd runs descending)
+  unsigned int* zero;  // if set, block 0 zeroes zero[0, nzero) (the next launch's progress flags)
+  int nzero;
 };
 
 // One merge group: A = src[a_off, a_off+na), B = src[b_off, b_off+nb),
@@ -71,6 +73,16 @@ struct MergeArgs {
   // bcf_merge_runs_u32 pass 1: B runs reversed into temp); nullptr = same
   const uint32_t* src_kb;
   const uint32_t* src_vb;
+  // multi-pass mode (persistent window kernel, regular passes only): npass
+  // consecutive passes in one launch.  Pass p reads buf_k[p & 1] (src_k is
+  // ignored), writes buf_k[(p + 1) & 1] or, for the last pass, dst_k; run
+  // length R << p, log2_tpg + p; decode_f32 applies to the last pass.  Pass p
+  // of a CTA starts once every CTA whose tiles cover its input groups has
+  // published progress[cta] >= p (zeroed before the launch).
+  int npass;
+  unsigned int* progress;
+  uint32_t* buf_k[2];
+  uint32_t* buf_v[2];
 };
 
 // Group of output tile `tile`: regular pairwise pass (run 2g with run 2g+1,
@@ -194,6 +206,9 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortA
   const long long rem = args.n - t0;
   const int cnt = rem < T ? (int)rem : T;
   tma::pdl_wait();  // the input may be produced by the preceding grid
+  // (after the wait: the preceding grid may be a merge launch using the flags)
+  if (args.zero != nullptr && tile == 0)
+    for (int k = tid; k < args.nzero; k += U) args.zero[k] = 0u;
 
   // keys only, E = 31: levels 0..4 (runs up to one warp) run in registers
   // across the warp (warp_bitonic_levels); any assignment of the warp's 992

@@ -18,6 +18,7 @@ struct Variant {
   MergeFn merge_table = nullptr;  // group-table pass, all runs ascending (CF)
   MergeFn merge_tma = nullptr;    // persistent TMA pass (CF, E coprime with 32); grid arg = tiles
   MergeFn merge_win = nullptr;    // the persistent window kernel itself (keys or pairs; reads src_kb/src_vb), or nullptr
+  MergeFn merge_multi = nullptr;  // the window kernel running MergeArgs::npass regular passes in one launch
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]

@@ -108,6 +108,25 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
   long long t_begin, t_end;
   cta_tile_range(tiles, per_cta, t_begin, t_end);
   if (t_end <= t_begin) return;
+  // multi-pass mode: passes p = 0..npass-1 of a sort in this one launch
+  // (MergeArgs::npass); a CTA keeps its tile range in every pass
+  const bool multi = args.npass > 1;
+  const int npass = multi ? args.npass : 1;
+  auto pass_args = [&](int p) {
+    MergeArgs a = args;
+    if (multi) {
+      const bool last = p == npass - 1;
+      a.src_k = args.buf_k[p & 1];
+      a.src_v = args.buf_v[p & 1];
+      a.dst_k = last ? args.dst_k : args.buf_k[(p + 1) & 1];
+      a.dst_v = last ? args.dst_v : args.buf_v[(p + 1) & 1];
+      a.R = args.R << p;
+      a.log2_tpg = args.log2_tpg + p;
+      a.decode_f32 = last ? args.decode_f32 : 0;
+      a.trace = nullptr;
+    }
+    return a;
+  };
   // stage s: SW key words, then (pairs) SW value words at the same offsets
   auto stage = [&](int s) { return smem_dyn + (size_t)s * SW * (PAIRS ? 2 : 1); };
   auto stage_v = [&](int s) { return smem_dyn + (size_t)s * SW * (PAIRS ? 2 : 1) + SW; };
@@ -125,6 +144,34 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
 
   if (warp == NW) {
     // =========================== producer ===========================
+    // the CTA owning tile t (inverse of cta_tile_range with per_cta = 0)
+    auto cta_of_tile = [&](long long t) {
+      const long long G = gridDim.x;
+      long long c = (t * G) / tiles;
+      while (c + 1 < G && ((c + 1) * tiles) / G <= t) ++c;
+      while (c > 0 && (c * tiles) / G > t) --c;
+      return c;
+    };
+    int i = 0;  // ring index over every subtile and pass-end marker of the launch
+    for (int p = 0; p < npass; ++p) {
+    const MergeArgs args = pass_args(p);  // shadows the launch arguments inside the pass
+    if (p > 0) {
+      // pass p reads the groups of pass p-1 that its tiles fall in: wait until
+      // every CTA covering them has published pass p-1, then order the bulk
+      // copies below after those acquires
+      const int l = args.log2_tpg;
+      const long long gb = (t_begin >> l) << l;
+      long long ge = (((t_end - 1) >> l) + 1) << l;
+      if (ge > tiles) ge = tiles;
+      const long long c_lo = cta_of_tile(gb), c_hi = cta_of_tile(ge - 1);
+      for (;;) {
+        bool ok = true;
+        for (long long c = c_lo + lane; c <= c_hi; c += W) ok = ok && tma::ld_acquire_gpu(args.progress + c) >= (unsigned)p;
+        if (__all_sync(FULL, ok)) break;
+        __nanosleep(64);
+      }
+      tma::fence_proxy_async_global();
+    }
     const uint32_t* __restrict__ src = args.src_k;
     // B runs (table mode, bcf_merge_u32): a separate base, stored descending
     const uint32_t* __restrict__ srcB = args.src_kb ? args.src_kb : args.src_k;
@@ -146,8 +193,8 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
     long long D0 = j0 * T;
     long long a0;
     {
-      RunView Av{src + grp.a_off, grp.na, 0};
-      RunView Bv{srcB + grp.b_off, grp.nb, 1};
+      RunView Av{src + grp.a_off, grp.na, 0, multi ? 1 : 0};
+      RunView Bv{srcB + grp.b_off, grp.nb, 1, multi ? 1 : 0};
       const long long lenG = grp.na + grp.nb;
       const long long guess = lenG > 0 ? (long long)((double)D0 * (double)grp.na / (double)lenG) : 0;
       a0 = j0 == 0 ? 0 : merge_path_warp_global_guess(Av, Bv, D0, 0, D0, guess, lane);
@@ -249,8 +296,11 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         pb0 = (pb0 + 3) & ~3ll;
         if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
       }
-      const uint32_t ev = w >= 0 ? __ldg(esrc + gw) : 0u;
-      const uint32_t evv = (PAIRS && w >= 0) ? __ldg(esrcv + gw) : 0u;
+      uint32_t ev = 0u, evv = 0u;
+      if (w >= 0) {
+        ev = multi ? ld_cg(esrc + gw) : __ldg(esrc + gw);
+        if constexpr (PAIRS) evv = multi ? ld_cg(esrcv + gw) : __ldg(esrcv + gw);
+      }
       // lane 0 stores the <= 6 edge words itself, then release-arrives: the
       // stores precede the arrive in one thread's program order (a lane-l
       // store ordered only through __syncwarp is invisible to racecheck)
@@ -299,13 +349,14 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       }
     };
 
-    load_window(0);
+    const int i0 = i;
+    load_window(i % S);
     if (lane == 0) BCF_TRACE_AT(128 + 2);
-    for (int i = 0;; ++i) {
+    for (;; ++i) {
       const int s = i % S;
       const int s1 = (i + 1) % S;      // stage of the next window
       const int sp = (i + S - 1) % S;  // stage of subtile i-1 (= s1 for 2 stages)
-      if (i >= 1) {
+      if (i >= i0 + 1) {
         // subtile i-1's outputs are staged in sp: stream them out while the
         // consumers search subtile i's split
         tma::mbar_wait(&empty_bar[sp], (uint32_t)((i - 1) / S) & 1);
@@ -340,6 +391,20 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         store_out(s);
         if (lane == 0) tma::bulk_wait_all();
         __syncwarp();
+        if (multi) {
+          // the consumers acknowledge the pass-end marker on its split and
+          // empty barriers (every barrier of a stage stays in phase), then
+          // this CTA's outputs of pass p are published
+          tma::mbar_wait(&split_bar[s1], (uint32_t)((i + 1) / S) & 1);
+          tma::mbar_wait(&empty_bar[s1], (uint32_t)((i + 1) / S) & 1);
+          if (lane == 0) {
+            tma::fence_proxy_async_global();
+            __threadfence();
+            tma::st_release_gpu(args.progress + blockIdx.x, (unsigned)(p + 1));
+          }
+          __syncwarp();
+        }
+        i += 2;  // the last subtile and the marker
         break;
       }
       // stage s1's last store (subtile i+1-S) has read it: with 2 stages that
@@ -352,19 +417,30 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       load_window(s1);
       if (lane == 0 && i < 6) BCF_TRACE_AT(128 + 4 * (i + 1) + 2);
     }
+    }  // passes
     return;
   }
 
   // ============================ consumers ============================
-  const bool decode = args.decode_f32 != 0;
   uint32_t val[E];  // values (pairs); unused for keys
-  for (int i = 0;; ++i) {
+  int i = 0;
+  for (int p = 0; p < npass; ++p) {
+  const MergeArgs args = pass_args(p);
+  const bool decode = args.decode_f32 != 0;
+  for (;; ++i) {
     const int s = i % S;
     if (tid == 0 && i < 31) BCF_TRACE_AT(1 + 4 * i);
     tma::mbar_wait(&full_bar[s], (uint32_t)(i / S) & 1);
     if (tid == 0 && i < 31) BCF_TRACE_AT(2 + 4 * i);
     const WinMeta M = meta[s];
-    if (M.exit) break;
+    if (M.exit) {
+      if (multi && tid == 0) {
+        tma::mbar_arrive(&split_bar[s]);
+        tma::mbar_arrive(&empty_bar[s]);
+      }
+      ++i;
+      break;
+    }
     uint32_t* sk = stage(s) + M.c;  // logical index -> sk[index]
     uint32_t* sv = stage_v(s) + M.c;
     const int WA = M.WA, WB = M.WB, cmax = M.cmax;
@@ -467,11 +543,13 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         gb[ew] = sb[ew];
         if constexpr (PAIRS) args.dst_v[(M.c0 - M.cout) + ew] = stage_v(s)[ew];
       }
+      if (multi) __threadfence();  // edge words visible before the producer publishes the pass
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&empty_bar[s]);
     }
     if (tid == 0 && i < 31) BCF_TRACE_AT(3 + 4 * i);
   }
+  }  // passes
 }
 
 }  // namespace bcf

@@ -152,6 +152,14 @@ cudaError_t launch_merge_win(const MergeArgs& a, long long tiles, cudaStream_t s
                            s);
 }
 
+// every regular pass of a sort in one launch (MergeArgs::npass, progress flags)
+template <int E, int U, bool PAIRS>
+cudaError_t launch_merge_multi(const MergeArgs& a, long long tiles, cudaStream_t s) {
+  static PersistentCache pc;
+  return launch_persistent(merge_pass_win_kernel<E, U, PAIRS>, pc, win_smem_bytes<E, U, PAIRS>(), U + 32, a, tiles,
+                           s);
+}
+
 template <int E, int U>
 void register_eu(LaunchTable& t) {
   const int ui = u_index(U);
@@ -164,10 +172,14 @@ void register_eu(LaunchTable& t) {
   if constexpr (cgcd(W, E) == 1) {
     t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
     t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;
-    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024) {
       t.v[E][ui][0][0].merge_win = &launch_merge_win<E, U, false>;
-    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
+      t.v[E][ui][0][0].merge_multi = &launch_merge_multi<E, U, false>;
+    }
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024) {
       t.v[E][ui][0][1].merge_win = &launch_merge_win<E, U, true>;
+      t.v[E][ui][0][1].merge_multi = &launch_merge_multi<E, U, true>;
+    }
   }
 }
 
