@@ -151,25 +151,42 @@ static int trace_pass_wanted() {
   return want;
 }
 static bool trace_requested() { return trace_pass_wanted() >= 0; }
-static unsigned long long* trace_for_pass(int pass) {
-  if (pass != trace_pass_wanted()) return nullptr;
+// BCF_TRACE_MULTI=1: per-CTA, per-pass timeline of the multi-pass launch
+// (slots 4p: wait start, 4p+1: inputs ready, 4p+2: pass published)
+static unsigned long long* trace_buffer();
+static unsigned long long* multi_trace() {
+  static const bool on = [] {
+    const char* v = getenv("BCF_TRACE_MULTI");
+    return v && v[0] == '1';
+  }();
+  return on ? trace_buffer() : nullptr;
+}
+static unsigned long long* trace_buffer() {
   if (!g_trace) {
     if (cudaMalloc(&g_trace, TRACE_WORDS * 8) != cudaSuccess) return nullptr;
     cudaMemset(g_trace, 0, TRACE_WORDS * 8);
   }
   return g_trace;
 }
+static unsigned long long* trace_for_pass(int pass) {
+  if (pass != trace_pass_wanted()) return nullptr;
+  return trace_buffer();
+}
 
-// BCF_NO_MULTI=1: one launch per merge pass instead of every pass of a sort in
-// one persistent launch (A/B measurements)
+// BCF_MULTI=1: every merge pass of a sort in one persistent launch (dataflow
+// between passes through per-CTA progress flags) instead of one launch per
+// pass.  Off by default: measured slower at 2^24 (0.551 vs 0.517 ms per sort,
+// profiles/r02_trace_multipass_2p24.txt): per-CTA pass times vary ~2.5x and
+// the dependency chains accumulate that spread, while the per-pass launches
+// overlap through PDL.
 static bool multipass_disabled() {
   static const bool off = [] {
-    const char* v = getenv("BCF_NO_MULTI");
-    return v && v[0] == '1';
+    const char* v = getenv("BCF_MULTI");
+    return !(v && v[0] == '1');
   }();
   return off;
 }
-static constexpr int MAX_PROGRESS_CTAS = 2048;
+static constexpr int MAX_PROGRESS_CTAS = 2048;  // 1536 per-CTA flags + 512 per-pass counters
 
 // BCF_NO_TMA=1 selects the non-persistent merge kernel (A/B measurements)
 static bool tma_disabled() {
@@ -256,6 +273,7 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
     ma.buf_k[1] = Y;
     ma.buf_v[0] = XV;
     ma.buf_v[1] = YV;
+    ma.trace = multi_trace();
     e = launch("merge_passes", n * (uint64_t)P, s, [&] { return var.merge_multi(ma, tiles, s); });
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }

@@ -65,7 +65,7 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // debug timeline: 256 slots per CTA (consumers at 1 + 4i, producer at 128 + 4i)
 #define BCF_TRACE_AT(slot)                                                          \
   do {                                                                              \
-    if (args.trace && (slot) < 256) args.trace[(size_t)blockIdx.x * 256 + (slot)] = gtimer(); \
+    if (args.trace && args.npass <= 1 && (slot) < 256) args.trace[(size_t)blockIdx.x * 256 + (slot)] = gtimer(); \
   } while (0)
 
 // tiles [t_begin, t_end) of this CTA: per_cta > 0 -> fixed chunks of per_cta

@@ -46,6 +46,10 @@ __host__ __device__ constexpr size_t win_smem_bytes() {
   return (size_t)WIN_STAGES * win_stage_words<E, U>() * sizeof(uint32_t) * (PAIRS ? 2 : 1);
 }
 
+// progress words of a multi-pass launch: per-CTA flags at [0, MULTI_COUNTERS_AT),
+// then one completed-CTA counter per pass
+constexpr int MULTI_COUNTERS_AT = 1536;
+
 struct WinMeta {
   long long c0;       // output global word of logical output index q
   int WA, WB;         // window sizes (keys of A / B present)
@@ -123,7 +127,6 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       a.R = args.R << p;
       a.log2_tpg = args.log2_tpg + p;
       a.decode_f32 = last ? args.decode_f32 : 0;
-      a.trace = nullptr;
     }
     return a;
   };
@@ -164,13 +167,23 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       long long ge = (((t_end - 1) >> l) + 1) << l;
       if (ge > tiles) ge = tiles;
       const long long c_lo = cta_of_tile(gb), c_hi = cta_of_tile(ge - 1);
-      for (;;) {
-        bool ok = true;
-        for (long long c = c_lo + lane; c <= c_hi; c += W) ok = ok && tma::ld_acquire_gpu(args.progress + c) >= (unsigned)p;
-        if (__all_sync(FULL, ok)) break;
-        __nanosleep(64);
+      if (lane == 0 && args.trace) args.trace[(size_t)blockIdx.x * 256 + 4 * p] = gtimer();
+      if (c_hi - c_lo + 1 >= (long long)gridDim.x) {
+        // every CTA: the pass counter (one word) instead of G flags
+        const unsigned* cnt = args.progress + MULTI_COUNTERS_AT + (p - 1);
+        while (tma::ld_acquire_gpu(cnt) < gridDim.x) __nanosleep(200);
+      } else {
+        for (;;) {
+          bool ok = true;
+          for (long long c = c_lo + lane; c <= c_hi; c += W)
+            ok = ok && tma::ld_acquire_gpu(args.progress + c) >= (unsigned)p;
+          if (__all_sync(FULL, ok)) break;
+          __nanosleep(200);
+        }
       }
+      __syncwarp();
       tma::fence_proxy_async_global();
+      if (lane == 0 && args.trace) args.trace[(size_t)blockIdx.x * 256 + 4 * p + 1] = gtimer();
     }
     const uint32_t* __restrict__ src = args.src_k;
     // B runs (table mode, bcf_merge_u32): a separate base, stored descending
@@ -401,6 +414,8 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
             tma::fence_proxy_async_global();
             __threadfence();
             tma::st_release_gpu(args.progress + blockIdx.x, (unsigned)(p + 1));
+            atomicAdd(args.progress + MULTI_COUNTERS_AT + p, 1u);  // pass counter (after the fence)
+            if (args.trace) args.trace[(size_t)blockIdx.x * 256 + 4 * p + 2] = gtimer();
           }
           __syncwarp();
         }
@@ -543,7 +558,6 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         gb[ew] = sb[ew];
         if constexpr (PAIRS) args.dst_v[(M.c0 - M.cout) + ew] = stage_v(s)[ew];
       }
-      if (multi) __threadfence();  // edge words visible before the producer publishes the pass
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(&empty_bar[s]);
     }
