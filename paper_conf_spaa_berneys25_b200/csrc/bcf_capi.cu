@@ -188,11 +188,31 @@ static bool multipass_disabled() {
 }
 static constexpr int MAX_PROGRESS_CTAS = 2048;  // 1536 per-CTA flags + 512 per-pass counters
 
+// BCF_ONE_CTA_PER_SM=1 (measurement mode for the unit-level bank-conflict
+// counter): LSU-only kernels (block sort and the plain merge kernel, no bulk
+// copies) with one CTA per SM looping over tiles.  ncu's
+// l1tex__data_bank_conflicts_pipe_lsu_mem_shared also counts ~6 store
+// wavefronts per CTA launched onto an SM that runs other CTAs, and port
+// arbitration between STS and async copies (tools/ncu_calib_lsu.cu); this mode
+// has neither, so the counter measures address conflicts alone.
+static bool one_cta_per_sm() {
+  static const bool on = [] {
+    const char* v = getenv("BCF_ONE_CTA_PER_SM");
+    return v && v[0] == '1';
+  }();
+  return on;
+}
+static long long sm_count() {
+  int dev = 0, sms = 148;
+  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return sms;
+}
+
 // BCF_NO_TMA=1 selects the non-persistent merge kernel (A/B measurements)
 static bool tma_disabled() {
   static const bool off = [] {
     const char* v = getenv("BCF_NO_TMA");
-    return v && v[0] == '1';
+    return (v && v[0] == '1') || one_cta_per_sm();
   }();
   return off;
 }
@@ -263,7 +283,13 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   // the block sort zeroes the progress flags (no memset between the two launches)
   SortArgs sa{in_k, in_v, P == 0 ? out_k : X, P == 0 ? out_v : XV, (long long)n, f32 ? 1 : 0,
               (f32 && P == 0) ? 1 : 0, cf ? 1 : 0, multi ? progress : nullptr, multi ? MAX_PROGRESS_CTAS : 0};
-  cudaError_t e = launch("block_sort", n, s, [&] { return vbs.block_sort(sa, tiles_bs, s); });
+  const bool one_sm = one_cta_per_sm();
+  long long grid_bs = tiles_bs;
+  if (one_sm && tiles_bs > sm_count()) {
+    grid_bs = sm_count();
+    sa.ntiles = tiles_bs;
+  }
+  cudaError_t e = launch("block_sort", n, s, [&] { return vbs.block_sort(sa, grid_bs, s); });
   if (e != cudaSuccess) return cuda_fail(e);
   if (multi) {
     MergeArgs ma{X, XV, out_k, out_v, (long long)n, Tbs, 1 + lg_bs, f32 ? 1 : 0, cf ? 1 : 0, nullptr, 0, nullptr};
@@ -288,10 +314,15 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
     // (the keys'): a final pass into key / value outputs of different phases
     // takes the plain kernel
     const bool phase_ok = !pairs || i < P || (((uintptr_t)out_k ^ (uintptr_t)out_v) & 15) == 0;
+    long long grid = tiles;
+    if (one_sm && tiles > sm_count()) {
+      grid = sm_count();
+      ma.ntiles = tiles;
+    }
     if (use_tma && phase_ok)
       e = launch("merge_pass", n, s, [&] { return var.merge_tma(ma, tiles, s); });
     else
-      e = launch("merge_pass", n, s, [&] { return var.merge(ma, tiles, s); });
+      e = launch("merge_pass", n, s, [&] { return var.merge(ma, grid, s); });
     if (e != cudaSuccess) return cuda_fail(e);
   }
   return BCF_SUCCESS;

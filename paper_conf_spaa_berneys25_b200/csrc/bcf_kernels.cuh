@@ -46,6 +46,7 @@ struct SortArgs {
   int cf_dirs;     // CF run directions (odd runs descending)
   unsigned int* zero;  // if set, block 0 zeroes zero[0, nzero) (the next launch's progress flags)
   int nzero;
+  long long ntiles;    // > 0: a grid smaller than the tile count loops over tiles (grid stride)
 };
 
 // One merge group: A = src[a_off, a_off+na), B = src[b_off, b_off+nb),
@@ -83,6 +84,7 @@ struct MergeArgs {
   unsigned int* progress;
   uint32_t* buf_k[2];
   uint32_t* buf_v[2];
+  long long ntiles;  // plain kernel: > 0 -> grid-stride loop over this many tiles
 };
 
 // Group of output tile `tile`: regular pairwise pass (run 2g with run 2g+1,
@@ -191,7 +193,7 @@ __host__ __device__ constexpr int bs_min_blocks() {
 }
 
 template <int E, int U, bool PAIRS, bool CF>
-__global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortArgs args) {
+__device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long long tile) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
   extern __shared__ __align__(16) uint32_t smem_dyn[];
@@ -201,7 +203,6 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortA
   const int tid = threadIdx.x;
   const int lane = tid & (W - 1);
   const int warp = tid >> 5;
-  const long long tile = blockIdx.x;
   const long long t0 = tile * T;
   const long long rem = args.n - t0;
   const int cnt = rem < T ? (int)rem : T;
@@ -393,8 +394,17 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortA
 // Merge pass (K2+K3 fused): output tile `blockIdx.x` of the pairwise merge of
 // runs of R keys.  Group g merges run 2g (A) with run 2g+1 (B).
 // ---------------------------------------------------------------------------
+template <int E, int U, bool PAIRS, bool CF>
+__global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortArgs args) {
+  const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
+  for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
+    if (t != blockIdx.x) __syncthreads();  // the previous tile's copy-out has read shared memory
+    block_sort_tile<E, U, PAIRS, CF>(args, t);
+  }
+}
+
 template <int E, int U, bool PAIRS, bool CF, bool BDESC>
-__global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
+__device__ __forceinline__ void merge_pass_tile(const MergeArgs& args, const long long tile) {
   constexpr int T = U * E;
   constexpr int NW = U / W;
   extern __shared__ __align__(16) uint32_t smem_dyn[];
@@ -405,7 +415,6 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   const int tid = threadIdx.x;
   const int lane = tid & (W - 1);
   const int warp = tid >> 5;
-  const long long tile = blockIdx.x;
   tma::pdl_wait();  // pass i reads what pass i-1 wrote (and overwrites what it read)
   long long j;
   const GroupDesc grp = group_of_tile(args, tile, T, j);
@@ -531,6 +540,15 @@ __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
   const long long c0 = desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
   store_tile<E, U, PAIRS>(sk, sv, key, val, D, cnt, desc, args.dst_k, args.dst_v, c0,
                           args.decode_f32 != 0);
+}
+
+template <int E, int U, bool PAIRS, bool CF, bool BDESC>
+__global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
+  const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
+  for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
+    if (t != blockIdx.x) __syncthreads();
+    merge_pass_tile<E, U, PAIRS, CF, BDESC>(args, t);
+  }
 }
 
 }  // namespace bcf

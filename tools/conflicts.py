@@ -33,7 +33,7 @@ def main():
     n = a.n
     x_rand = si.uniform_u32_torch(n, si.config_seed(1), dev)
     mapping = []
-    launch = bcf.launch_count()
+    seen = 0  # library launches of the sorts so far (the ncu -k filter drops the generator's)
     for cfg in a.configs.split(","):
         algo, E, u = cfg.split(":")
         E, u = int(E), int(u)
@@ -46,7 +46,8 @@ def main():
             torch.cuda.synchronize()
             last = bcf.launch_count()
             mapping.append({"algo": algo, "E": E, "u": u, "kind": kind, "n": n,
-                            "first_launch": first - launch, "launches": last - first})
+                            "first_launch": seen, "launches": last - first})
+            seen += last - first
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(mapping, f, indent=1)
