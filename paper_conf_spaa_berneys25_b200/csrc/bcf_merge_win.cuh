@@ -35,7 +35,11 @@ __host__ __device__ constexpr int win_span() {
 }
 template <int E, int U>
 __host__ __device__ constexpr int win_stage_words() {
-  return ((win_span<E, U>() + E + 8) + 3) / 4 * 4;  // span + cell-scan slack + shift
+  // span + cell-scan slack + shift; with rho != identity the slack probes of
+  // logical words past the span land anywhere in the next rho partition
+  constexpr int d = cgcd(W, E);
+  constexpr int slack = (d > 1 && W * E / d > E + 8) ? W * E / d : E + 8;
+  return ((win_span<E, U>() + slack) + 3) / 4 * 4;
 }
 #ifndef BCF_WIN_STAGES
 #define BCF_WIN_STAGES 2
@@ -97,7 +101,11 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
   constexpr int NW = U / W;
   constexpr int SW = win_stage_words<E, U>();
   constexpr int S = WIN_STAGES;
-  static_assert(cgcd(W, E) == 1, "window staging needs rho = identity (E coprime with 32)");
+  // E sharing factors with w (d > 1, rho != identity, §3.2): the
+  // producer stages windows in rho's physical order with 4-byte cp.async
+  // (bulk copies cannot rotate 4-byte words inside a partition), the
+  // consumers copy the outputs out with LSU loads / stores
+  constexpr bool RHO = cgcd(W, E) > 1;
   static_assert(S2 % (W * E) == 0 && S2 % 4 == 0 && S2 > T, "span must be a multiple of wE");
   extern __shared__ __align__(16) uint32_t smem_dyn[];
   __shared__ WinMeta meta[S];
@@ -136,7 +144,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
-      tma::mbar_init(&full_bar[s], 1);
+      tma::mbar_init(&full_bar[s], RHO ? 32 : 1);
       tma::mbar_init(&empty_bar[s], 1);
       tma::mbar_init(&split_bar[s], 1);
     }
@@ -243,14 +251,55 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       M.exit = 0;
       const long long oA = grp.a_off + a0;                  // A[a0 + q] at word oA + q
       const long long oB = grp.b_off + grp.nb - b0 - S2;    // logical q (B part) at oB + q
-      const int c = (int)(oA & 3);
+      const int c = RHO ? 0 : (int)(oA & 3);
       M.c = c;
       M.desc = grp.out_desc;
       M.c0 = M.desc ? grp.out_off + lenG - D0 - T : grp.out_off + D0;
-      M.cout = (int)((unsigned long long)(dst_phase + M.c0) & 3ull);
+      M.cout = RHO ? 0 : (int)((unsigned long long)(dst_phase + M.c0) & 3ull);
       M.NA = 0;
       M.cnt = 0;
       if (lane == 0) meta[s] = M;
+      auto prefetch_next = [&]() {
+        // L2 prefetch of the keys the next window will need beyond this one
+        // (both runs are consumed sequentially): the next window's loads,
+        // issued one subtile later, then hit L2 instead of DRAM
+        constexpr long long PF = (3 * T / 4 + 3) & ~3;
+        const long long pa0 = (oA + WA + 3) & ~3ll;                  // A: ascending words
+        long long pa1 = grp.a_off + grp.na;
+        if (pa1 > pa0 + PF) pa1 = pa0 + PF;
+        pa1 &= ~3ll;
+        if (pa1 > pa0) tma::bulk_prefetch_l2(src + pa0, (uint32_t)(pa1 - pa0) * 4u);
+        long long pb1 = (grp.b_off + grp.nb - b0 - WB) & ~3ll;      // B: descending words
+        long long pb0 = grp.b_off;
+        if (pb0 < pb1 - PF) pb0 = pb1 - PF;
+        pb0 = (pb0 + 3) & ~3ll;
+        if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
+      };
+      if constexpr (RHO) {
+        // logical word q of the window at physical slot rho(q): A from
+        // src[oA + q] (q < WA), B from srcB[oB + q] (q >= S2 - WB); one
+        // warp-wide 4-byte cp.async per 32 consecutive words (coalesced
+        // reads, rotated conflict-free writes)
+        __syncwarp();  // meta[s] written before any lane's copies land
+        uint32_t* sk = stage(s);
+        for (int q = lane; q < WA; q += W) {
+          tma::cp_async4(sk + rho<E>(q), src + oA + q);
+          if constexpr (PAIRS) tma::cp_async4(stage_v(s) + rho<E>(q), srcv + oA + q);
+        }
+        for (int q = S2 - WB + lane; q < S2; q += W) {
+          tma::cp_async4(sk + rho<E>(q), srcB + oB + q);
+          if constexpr (PAIRS) tma::cp_async4(stage_v(s) + rho<E>(q), srcvB + oB + q);
+        }
+        if (lane == 0) {
+          prefetch_next();
+          tma::cp_async_wait_all();          // lane 0: its copies, then a release arrive (meta)
+          tma::mbar_arrive(&full_bar[s]);
+        } else {
+          tma::cp_async_mbar_arrive_noinc(&full_bar[s]);  // when this lane's copies have landed
+        }
+        __syncwarp();
+        return;
+      }
       int a_hi = WA ? align_up4(c + WA) : 0;
       int b_lo = WB ? align_dn4(c + S2 - WB) : 0;
       const int b_hi = WB ? align_up4(c + S2) : 0;
@@ -294,20 +343,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
           if (b_hi > b_lo)
             tma::bulk_g2s(sv + b_lo, srcvB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
         }
-        // L2 prefetch of the keys the next window will need beyond this one
-        // (both runs are consumed sequentially): the next window's bulk loads,
-        // issued one subtile later, then hit L2 instead of DRAM
-        constexpr long long PF = (3 * T / 4 + 3) & ~3;
-        const long long pa0 = (oA + WA + 3) & ~3ll;                  // A: ascending words
-        long long pa1 = grp.a_off + grp.na;
-        if (pa1 > pa0 + PF) pa1 = pa0 + PF;
-        pa1 &= ~3ll;
-        if (pa1 > pa0) tma::bulk_prefetch_l2(src + pa0, (uint32_t)(pa1 - pa0) * 4u);
-        long long pb1 = (grp.b_off + grp.nb - b0 - WB) & ~3ll;      // B: descending words
-        long long pb0 = grp.b_off;
-        if (pb0 < pb1 - PF) pb0 = pb1 - PF;
-        pb0 = (pb0 + 3) & ~3ll;
-        if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
+        prefetch_next();
       }
       uint32_t ev = 0u, evv = 0u;
       if (w >= 0) {
@@ -331,10 +367,9 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       if (lane == 0) tma::mbar_arrive(&full_bar[s]);
     };
     auto post_exit = [&](int s) {
-      if (lane == 0) {
-        meta[s].exit = 1;
-        tma::mbar_arrive(&full_bar[s]);
-      }
+      if (lane == 0) meta[s].exit = 1;
+      __syncwarp();
+      if (RHO || lane == 0) tma::mbar_arrive(&full_bar[s]);  // RHO: 32 arrivals per phase
       __syncwarp();
     };
 
@@ -348,6 +383,7 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
     // 16-byte aligned middle; warp 0 of the consumers writes the <= 7 + 3
     // edge words).  Issued and waited on by lane 0 (bulk groups are per thread).
     auto store_out = [&](int s) {
+      if constexpr (RHO) return;  // the consumers copy the outputs out
       const WinMeta M = meta[s];
       const int qlo = M.desc ? T - M.cnt : 0, qhi = M.desc ? T : M.cnt;
       const int w0 = M.cout + qlo, w1 = M.cout + qhi;
@@ -472,13 +508,13 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       int cnt = cmax;
       if (!(M.fin & 1) && r == WA) {
         // A window exhausted at D_A = WA + #{B[y] < A[WA-1]} (ties go to A)
-        const uint32_t v = sk[WA - 1];
-        const int nb = warp_prefix_count(WB, [&](int y) { return sk[S2 - 1 - y] < v; }, lane);
+        const uint32_t v = lds<E>(sk, WA - 1);
+        const int nb = warp_prefix_count(WB, [&](int y) { return lds<E>(sk, S2 - 1 - y) < v; }, lane);
         cnt = WA + nb;
       } else if (!(M.fin & 2) && cmax - r == WB) {
         // B window exhausted at D_B = WB + #{A[x] <= B[WB-1]}
-        const uint32_t v = sk[S2 - WB];
-        const int na = warp_prefix_count(WA, [&](int x) { return !(v < sk[x]); }, lane);
+        const uint32_t v = lds<E>(sk, S2 - WB);
+        const int na = warp_prefix_count(WA, [&](int x) { return !(v < lds<E>(sk, x)); }, lane);
         cnt = WB + na;
       }
       if (cnt < cmax) {
@@ -523,18 +559,41 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
     if (tid == 0 && i < 30) BCF_TRACE_AT(160 + 3 * i);
     uint32_t* ok = stage(s) + M.cout;
     uint32_t* ov = stage_v(s) + M.cout;
+    // round m of the staging writes logical D + m (or its mirror): a round
+    // set, conflict-free through rho (identity for E coprime with w)
     if (M.desc) {
 #pragma unroll
       for (int q = 0; q < E; ++q) {
-        ok[T - E - D + q] = key[E - 1 - q];
-        if constexpr (PAIRS) ov[T - E - D + q] = val[E - 1 - q];
+        ok[rho<E>(T - E - D + q)] = key[E - 1 - q];
+        if constexpr (PAIRS) ov[rho<E>(T - E - D + q)] = val[E - 1 - q];
       }
     } else {
 #pragma unroll
       for (int q = 0; q < E; ++q) {
-        ok[D + q] = key[q];
-        if constexpr (PAIRS) ov[D + q] = val[q];
+        ok[rho<E>(D + q)] = key[q];
+        if constexpr (PAIRS) ov[rho<E>(D + q)] = val[q];
       }
+    }
+    if constexpr (RHO) {
+      // LSU copy-out: physical slot P (consecutive per warp, conflict-free)
+      // holds logical output w = rho^-1(P), bound for global word c0 + w
+      tma::named_bar_sync(1, U);
+      const int qlo = M.desc ? T - cnt : 0;
+      const int qhi = M.desc ? T : cnt;
+      uint32_t* __restrict__ gk = args.dst_k + M.c0;
+      uint32_t* __restrict__ gv = PAIRS ? args.dst_v + M.c0 : nullptr;
+#pragma unroll
+      for (int r = 0; r < E; ++r) {
+        const int P = tid + r * U;
+        const int w = rho_inv<E>(P);
+        if (w >= qlo && w < qhi) {
+          gk[w] = ok[P];
+          if constexpr (PAIRS) gv[w] = ov[P];
+        }
+      }
+      tma::named_bar_sync(1, U);  // every consumer has read the stage
+      if (tid == 0) tma::mbar_arrive(&empty_bar[s]);
+      continue;
     }
     tma::fence_proxy_async_smem();  // the producer's bulk store reads these words
     tma::named_bar_sync(1, U);

@@ -169,6 +169,14 @@ void register_eu(LaunchTable& t) {
                       &launch_merge<E, U, true, true, false>};
   t.v[E][ui][1][0] = {&launch_block_sort<E, U, false, false>, &launch_merge<E, U, false, false, false>,
                       nullptr};
+  if constexpr (cgcd(W, E) > 1) {
+    // rho != identity: the window kernel with cp.async staging in rho's
+    // physical order and LSU copy-out (regular passes and merge_runs passes)
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
+      t.v[E][ui][0][0].merge_tma = &launch_merge_win<E, U, false>;
+    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
+      t.v[E][ui][0][1].merge_tma = &launch_merge_win<E, U, true>;
+  }
   if constexpr (cgcd(W, E) == 1) {
     t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
     t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;
