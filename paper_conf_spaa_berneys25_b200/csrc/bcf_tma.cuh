@@ -38,8 +38,33 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
   return done != 0;
 }
 
+// try_wait with a suspend-time hint: the warp sleeps in the barrier until the
+// phase completes (or the hint, 10 ms, expires) instead of re-issuing the
+// test, which leaves issue slots to the other warps of the SM
+__device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t parity) {
+  uint32_t done;
+  asm volatile(
+      "{\n"
+      " .reg .pred p;\n"
+      " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2, %3;\n"
+      " selp.u32 %0, 1, 0, p;\n"
+      "}\n"
+      : "=r"(done)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(10000000u)
+      : "memory");
+  return done != 0;
+}
+
+#ifndef BCF_MBAR_SPIN
+#define BCF_MBAR_SPIN 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  while (!mbar_try_wait(bar, parity)) {
+  if (BCF_MBAR_SPIN) {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+  } else {
+    while (!mbar_try_wait_sleep(bar, parity)) {
+    }
   }
 }
 
