@@ -8,6 +8,10 @@ paper_conf_spaa_berneys25_b200 computes, written from the paper
     addrmap.py      pi, rho and Alg. 1's gather schedule (§3)
     dmm.py          DMM bank-conflict cost model + Thrust serial-merge address stream
     worstcase.py    Section 4 worst-case construction (S, T, Theorem 8) + composition
+    setops_oracle.c set union / intersection / difference / symmetric difference
+                    of two sorted sequences, multiset semantics of ISO C++
+                    [alg.set.operations] (the paper's "parallel scan of a pair of
+                    arrays", PAPER.md:380)
     cpu_baselines.cpp  std::stable_sort (1 core) and a std::thread parallel
                     stable mergesort (all cores): the further CPU baselines of
                     SURVEY.md §8(d), also a library cross-check of the oracle
@@ -32,6 +36,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "sort_oracle.c")
+_SRC_SET = os.path.join(_HERE, "setops_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -44,9 +49,10 @@ _cpp = None
 def build(force: bool = False) -> str:
     """Compile sort_oracle.c with gcc (plain C, -O2, single thread) and the
     CPU baselines with g++ (-O2, std::thread)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC),
+                                                                           os.path.getmtime(_SRC_SET)):
         subprocess.check_call(
-            ["gcc", "-O2", "-std=c99", "-shared", "-fPIC", "-o", _LIB, _SRC]
+            ["gcc", "-O2", "-std=c99", "-shared", "-fPIC", "-o", _LIB, _SRC, _SRC_SET]
         )
     if force or not os.path.exists(_CPP_LIB) or os.path.getmtime(_CPP_LIB) < os.path.getmtime(_CPP_SRC):
         subprocess.check_call(
@@ -97,6 +103,9 @@ def lib():
             f.restype = ctypes.c_int
         L.oracle_sort_pairs_u32.argtypes = [u32p, u32p, u32p, u32p, ctypes.c_uint64]
         L.oracle_sort_pairs_u32.restype = ctypes.c_int
+        L.oracle_set_op_u32.argtypes = [ctypes.c_int, u32p, ctypes.c_uint64, u32p, ctypes.c_uint64, u32p, u32p,
+                                         ctypes.POINTER(ctypes.c_uint64)]
+        L.oracle_set_op_u32.restype = ctypes.c_int
         L.oracle_f32_total_less.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
         L.oracle_f32_total_less.restype = ctypes.c_int
         _lib = L
@@ -133,6 +142,22 @@ def sort_pairs_u32(keys: np.ndarray, vals: np.ndarray):
     if lib().oracle_sort_pairs_u32(_p(k), _p(v), _p(ko), _p(vo), k.size) != 0:
         raise MemoryError("oracle_sort_pairs_u32")
     return ko, vo
+
+
+SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}
+
+
+def set_op_u32(op: str, a: np.ndarray, b: np.ndarray):
+    """(keys, sources) of the set operation `op` on ascending a and b
+    (setops_oracle.c; source = A index, or 0x80000000 | B index)."""
+    a = np.ascontiguousarray(a, dtype=np.uint32)
+    b = np.ascontiguousarray(b, dtype=np.uint32)
+    out = np.empty(a.size + b.size + 1, dtype=np.uint32)
+    src = np.empty_like(out)
+    cnt = ctypes.c_uint64(0)
+    if lib().oracle_set_op_u32(SET_OPS[op], _p(a), a.size, _p(b), b.size, _p(out), _p(src), ctypes.byref(cnt)) != 0:
+        raise ValueError(op)
+    return out[:cnt.value].copy(), src[:cnt.value].copy()
 
 
 def f32_total_less(a: int, b: int) -> bool:
