@@ -178,6 +178,31 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
                          uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* p,
                          void* stream);
 
+/* Set operations of two ascending u32 sequences A = d_a[0, na) and
+   B = d_b[0, nb) with the multiset semantics of ISO C++ [alg.set.operations]:
+   for a key with m copies in A and n in B, union keeps all m copies from A
+   and then the last max(n - m, 0) of B's, intersection the first min(m, n)
+   of A's, difference (A - B) the last max(m - n, 0) of A's, symmetric
+   difference the last m - n of A's or the last n - m of B's.  The output is
+   ascending (equal keys: A's copies first).  The paper's generalisation of
+   its technique to "any algorithm that involves a parallel scan of a pair of
+   arrays": the pair is merged by the conflict-free merge
+   (bcf_merge_u32 with source tags, ties to A), then the kept elements of
+   every equal-key run are flagged and compacted in merged order.
+   d_out (na + nb words) receives the kept keys, d_out_src (optional, NULL
+   to skip) where each came from: the A index, or 0x80000000 | the B index;
+   *d_count (DEVICE u64) their number.  na, nb < 2^31.  Precondition: A and B
+   ascending (not checked).  Temp: CUB-style query. */
+typedef enum {
+  BCF_SET_UNION = 0,
+  BCF_SET_INTERSECTION = 1,
+  BCF_SET_DIFFERENCE = 2,
+  BCF_SET_SYMMETRIC_DIFFERENCE = 3
+} bcf_set_op;
+bcf_status bcf_set_op_u32(int32_t op, const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
+                          uint32_t* d_out, uint32_t* d_out_src, uint64_t* d_count, void* d_temp,
+                          size_t* temp_bytes, const bcf_params* p, void* stream);
+
 const char* bcf_status_string(bcf_status s);
 int32_t bcf_abi_version(void);
 /* cudaError_t (as int) of the last BCF_ERROR_CUDA on the calling thread */

@@ -11,6 +11,7 @@ calls raise.
     worst_case(n, E, u, seed)  Section 4 worst-case permutation (device tensor)
     worst_case_host(...)       same into a numpy array (no CUDA)
     merge(a, b)                stable merge of two sorted arrays (one CF merge pass)
+    set_op(op, a, b)           union / intersection / difference / symmetric difference
     split_counts, merge_runs   distributed-sort phases (see dist.py)
 """
 from __future__ import annotations
@@ -36,7 +37,7 @@ EXPORTED_SYMBOLS = [
     "bcf_default_params", "bcf_default_pairs_params", "bcf_sort_u32", "bcf_sort_f32", "bcf_sort_pairs_u32",
     "bcf_sort_u32_host_batch", "bcf_sort_plan", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_merge_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
-    "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy",
+    "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy", "bcf_set_op_u32",
 ]
 
 
@@ -101,6 +102,8 @@ def lib():
     L.bcf_profile_collect.argtypes = [P(KernelStats), i32, P(i32)]
     L.bcf_profile_collect.restype = ctypes.c_int
     L.bcf_launch_count.restype = ctypes.c_int64
+    L.bcf_set_op_u32.argtypes = [i32, vp, u64, vp, u64, vp, vp, vp, vp, P(ctypes.c_size_t), P(Params), vp]
+    L.bcf_set_op_u32.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -375,6 +378,41 @@ def merge(a, b, a_values=None, b_values=None, params: Params | None = None, out=
         _check(L.bcf_merge_u32(a.data_ptr(), a.numel(), b.data_ptr(), b.numel(), va, vb, out.data_ptr(), vo,
                                temp.data_ptr(), ctypes.byref(tb), pp, _stream(a)), "bcf_merge_u32")
     return (out, out_values) if a_values is not None else out
+
+
+SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}
+
+
+def set_op(op: str, a, b, with_source: bool = False, params: Params | None = None):
+    """Set operation of two ascending 1-D CUDA tensors of 4-byte keys (u32
+    order), multiset semantics of std::set_* (bcf_set_op_u32).  Returns the
+    kept keys (and, with_source, the int32 tags: A index or 0x80000000 | B
+    index).  Reads the output count back (synchronises the stream)."""
+    torch = _torch()
+    _require_cuda(a, "a")
+    _require_cuda(b, "b")
+    if b.device != a.device:
+        raise BcfError("a and b are on different devices")
+    if op not in SET_OPS:
+        raise BcfError(f"unknown set operation {op!r}")
+    n = a.numel() + b.numel()
+    out = torch.empty(max(1, n), dtype=a.dtype, device=a.device)
+    src = torch.empty(max(1, n), dtype=torch.int32, device=a.device) if with_source else None
+    cnt = torch.zeros(1, dtype=torch.int64, device=a.device)
+    L = lib()
+    pp = ctypes.byref(params) if params is not None else None
+    tb = ctypes.c_size_t(0)
+    _check(L.bcf_set_op_u32(SET_OPS[op], None, a.numel(), None, b.numel(), None, None, None, None,
+                            ctypes.byref(tb), pp, None), "temp query")
+    temp = _temp(tb.value, a.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(a.device):
+        _check(L.bcf_set_op_u32(SET_OPS[op], a.data_ptr() if a.numel() else None, a.numel(),
+                                b.data_ptr() if b.numel() else None, b.numel(), out.data_ptr(),
+                                src.data_ptr() if src is not None else None, cnt.data_ptr(), temp.data_ptr(),
+                                ctypes.byref(tb), pp, _stream(a)), "bcf_set_op_u32")
+    k = int(cnt.item())
+    return (out[:k], src[:k]) if with_source else out[:k]
 
 
 def profile_enable(on: bool = True):

@@ -17,6 +17,12 @@
 #include "bcf_launch.h"
 
 namespace bcf {
+namespace setops {
+cudaError_t make_tags(uint32_t* ta, long long na, uint32_t* tb, long long nb, cudaStream_t s);
+cudaError_t compact(int op, const uint32_t* M, const uint32_t* V, long long n, unsigned long long* counts,
+                    unsigned long long* d_count, uint32_t* out, uint32_t* out_src, cudaStream_t s);
+long long compact_blocks(long long n);
+}
 namespace wc {
 bool generate_host(uint32_t* out, uint64_t n, int E, int u, uint64_t seed);
 cudaError_t generate_device(uint32_t* out, uint64_t n, int E, int u, uint64_t seed, cudaStream_t s, bool* ok);
@@ -773,6 +779,47 @@ bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, 
   if (e != cudaSuccess) return cuda_fail(e);
   MergeArgs ma{d_a, d_a_vals, d_out, d_out_vals, (long long)n, 0, 0, 0, 0, dt, 1, nullptr, d_b, d_b_vals};
   e = launch("merge", n, s, [&] { return var.merge_table(ma, tiles, s); });
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
+bcf_status bcf_set_op_u32(int32_t op, const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
+                          uint32_t* d_out, uint32_t* d_out_src, uint64_t* d_count, void* d_temp, size_t* temp_bytes,
+                          const bcf_params* pp, void* stream) {
+  if (!temp_bytes || op < BCF_SET_UNION || op > BCF_SET_SYMMETRIC_DIFFERENCE) return BCF_ERROR_INVALID_VALUE;
+  if (na >= (1ull << 31) || nb >= (1ull << 31)) return BCF_ERROR_UNSUPPORTED;  // 31-bit source indices
+  const uint64_t n = na + nb;
+  // merge temp (pairs: keys + source tags)
+  size_t mtb = 0;
+  bcf_status st = bcf_merge_u32(nullptr, na, nullptr, nb, (const uint32_t*)16, (const uint32_t*)16, nullptr,
+                                (uint32_t*)16, nullptr, &mtb, pp, stream);
+  if (st != BCF_SUCCESS) return st;
+  const size_t ta_b = align_up(na * 4 + 4, 256), tb_b = align_up(nb * 4 + 4, 256), m_b = align_up(n * 4 + 4, 256);
+  const size_t c_b = align_up(((size_t)setops::compact_blocks((long long)n) + 1) * 8, 256);
+  const size_t need = 256 + ta_b + tb_b + 2 * m_b + c_b + mtb;
+  if (d_temp == nullptr) {
+    *temp_bytes = need;
+    return BCF_SUCCESS;
+  }
+  if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
+  if (!d_count || (n > 0 && !d_out) || (na && !d_a) || (nb && !d_b)) return BCF_ERROR_INVALID_VALUE;
+  cudaStream_t s = (cudaStream_t)stream;
+  char* tb = (char*)align_up((size_t)d_temp, 256);
+  uint32_t* ta = (uint32_t*)tb;
+  uint32_t* tbt = (uint32_t*)(tb + ta_b);
+  uint32_t* M = (uint32_t*)(tb + ta_b + tb_b);
+  uint32_t* V = (uint32_t*)(tb + ta_b + tb_b + m_b);
+  unsigned long long* counts = (unsigned long long*)(tb + ta_b + tb_b + 2 * m_b);
+  void* mt = tb + ta_b + tb_b + 2 * m_b + c_b;
+  cudaError_t e = launch("setop_tags", n, s, [&] { return setops::make_tags(ta, (long long)na, tbt, (long long)nb, s); });
+  if (e != cudaSuccess) return cuda_fail(e);
+  if (n > 0) {
+    size_t m2 = mtb;
+    st = bcf_merge_u32(d_a, na, d_b, nb, na ? ta : nullptr, nb ? tbt : nullptr, M, V, mt, &m2, pp, stream);
+    if (st != BCF_SUCCESS) return st;
+  }
+  e = launch("setop_compact", n, s, [&] {
+    return setops::compact(op, M, V, (long long)n, counts, (unsigned long long*)d_count, d_out, d_out_src, s);
+  });
   return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
 }
 

@@ -200,3 +200,23 @@ def test_sort_plan():
     assert bcf.sort_plan(1 << 26, bcf.make_params(17, 256), pairs=True)["merge_passes"] == 14
     assert bcf.sort_plan(1 << 24, bcf.make_params(15, 256)) == {"block_sort_tile": 3840, "merge_tile": 3840,
                                                                "merge_passes": 13}
+
+
+def test_set_op_query_and_validation():
+    """bcf_set_op_u32: CUB-style temp query and synchronous argument errors
+    (no GPU needed)."""
+    L = bcf.lib()
+    tb = ctypes.c_size_t(0)
+    assert L.bcf_set_op_u32(0, None, 1000, None, 2000, None, None, None, None, ctypes.byref(tb), None, None) == 0
+    assert tb.value >= 4 * 3000 * 2  # merged keys + tags at least
+    assert L.bcf_set_op_u32(4, None, 10, None, 10, None, None, None, None, ctypes.byref(tb), None,
+                            None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_set_op_u32(-1, None, 10, None, 10, None, None, None, None, ctypes.byref(tb), None,
+                            None) == bcf.BCF_ERROR_INVALID_VALUE
+    assert L.bcf_set_op_u32(0, None, 1 << 31, None, 10, None, None, None, None, ctypes.byref(tb), None,
+                            None) == bcf.BCF_ERROR_UNSUPPORTED
+    big = ctypes.c_size_t(1 << 40)
+    fake = ctypes.c_void_p(256)
+    # count pointer missing
+    assert L.bcf_set_op_u32(1, fake, 10, fake, 10, fake, None, None, fake, ctypes.byref(big), None,
+                            None) == bcf.BCF_ERROR_INVALID_VALUE
