@@ -147,6 +147,31 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
                               uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes,
                               const bcf_params* p, void* stream);
 
+/* bcf_merge_runs_u32 for runs anywhere in device memory, keys only: run r is
+   h_run_ptrs[r][0, h_run_lens[r]) (host arrays of nruns entries; the
+   pointers may be peer-mapped memory of other GPUs, bcf_ipc_open).  The
+   first pairwise pass reads every run through its own pointer (over NVLink
+   for a peer's run), so an all-to-all exchange followed by the run merge
+   becomes one pass that moves each key once; later
+   passes are local.  Equal keys keep run order (run 0 first).  nruns <= 4096.
+   Temp: CUB-style query, as bcf_merge_runs_u32 of the same lengths.  The
+   caller orders the producers of peer runs before this call (e.g. stream
+   synchronise + barrier) and keeps them alive until it completes. */
+bcf_status bcf_merge_runs_ptrs_u32(const uint32_t* const* h_run_ptrs, const uint64_t* h_run_lens,
+                                   int32_t nruns, uint32_t* d_out, void* d_temp, size_t* temp_bytes,
+                                   const bcf_params* p, void* stream);
+
+/* CUDA IPC for bcf_merge_runs_ptrs_u32 across the processes of one node
+   (one process per GPU).  bcf_ipc_export: the handle (BCF_IPC_HANDLE_BYTES
+   bytes written to `handle`) of the allocation holding d_ptr and d_ptr's
+   byte offset in it.  bcf_ipc_open: map a peer's handle (peer access enabled
+   lazily); *d_base = the allocation's base in this process.  bcf_ipc_close:
+   unmap. */
+#define BCF_IPC_HANDLE_BYTES 64
+bcf_status bcf_ipc_export(const void* d_ptr, void* handle, uint64_t* offset);
+bcf_status bcf_ipc_open(const void* handle, void** d_base);
+bcf_status bcf_ipc_close(void* d_base);
+
 /* Stable merge of two ascending sorted arrays A = d_a[0, na) and
    B = d_b[0, nb) into d_out[0, na+nb) (must alias neither); equal keys: all
    of A's before B's.  The merge step of the pairwise mergesort (merge path,

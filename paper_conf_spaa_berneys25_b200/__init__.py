@@ -38,6 +38,7 @@ EXPORTED_SYMBOLS = [
     "bcf_sort_u32_host_batch", "bcf_sort_plan", "bcf_worst_case_u32", "bcf_worst_case_u32_host", "bcf_split_counts_u32",
     "bcf_merge_runs_u32", "bcf_merge_u32", "bcf_status_string", "bcf_abi_version", "bcf_last_cuda_error",
     "bcf_profile_enable", "bcf_profile_collect", "bcf_launch_count", "bcf_debug_trace_copy", "bcf_set_op_u32",
+    "bcf_merge_runs_ptrs_u32", "bcf_ipc_export", "bcf_ipc_open", "bcf_ipc_close",
 ]
 
 
@@ -102,6 +103,14 @@ def lib():
     L.bcf_profile_collect.argtypes = [P(KernelStats), i32, P(i32)]
     L.bcf_profile_collect.restype = ctypes.c_int
     L.bcf_launch_count.restype = ctypes.c_int64
+    L.bcf_merge_runs_ptrs_u32.argtypes = [vp, vp, i32, vp, vp, P(sz), P(Params), vp]
+    L.bcf_merge_runs_ptrs_u32.restype = ctypes.c_int
+    L.bcf_ipc_export.argtypes = [vp, vp, P(u64)]
+    L.bcf_ipc_export.restype = ctypes.c_int
+    L.bcf_ipc_open.argtypes = [vp, P(vp)]
+    L.bcf_ipc_open.restype = ctypes.c_int
+    L.bcf_ipc_close.argtypes = [vp]
+    L.bcf_ipc_close.restype = ctypes.c_int
     L.bcf_set_op_u32.argtypes = [i32, vp, u64, vp, u64, vp, vp, vp, vp, P(ctypes.c_size_t), P(Params), vp]
     L.bcf_set_op_u32.restype = ctypes.c_int
     _lib = L
@@ -378,6 +387,51 @@ def merge(a, b, a_values=None, b_values=None, params: Params | None = None, out=
         _check(L.bcf_merge_u32(a.data_ptr(), a.numel(), b.data_ptr(), b.numel(), va, vb, out.data_ptr(), vo,
                                temp.data_ptr(), ctypes.byref(tb), pp, _stream(a)), "bcf_merge_u32")
     return (out, out_values) if a_values is not None else out
+
+
+def merge_runs_ptrs(run_ptrs, run_lens, device, dtype=None, params: Params | None = None, out=None):
+    """bcf_merge_runs_ptrs_u32: stable merge of sorted runs given as raw
+    device pointers (ints; local or peer-mapped) and lengths; returns a new
+    CUDA tensor on `device` (int32 unless dtype is given)."""
+    torch = _torch()
+    nr = len(run_ptrs)
+    if len(run_lens) != nr:
+        raise BcfError("run_ptrs and run_lens differ in length")
+    n = int(sum(int(x) for x in run_lens))
+    if out is None:
+        out = torch.empty(max(1, n), dtype=dtype or torch.int32, device=device)
+    _require_cuda(out, "out")
+    ptrs = (ctypes.c_void_p * max(1, nr))(*[int(p) for p in run_ptrs])
+    lens = (ctypes.c_uint64 * max(1, nr))(*[int(x) for x in run_lens])
+    L = lib()
+    pp = ctypes.byref(params) if params is not None else None
+    tb = ctypes.c_size_t(0)
+    _check(L.bcf_merge_runs_ptrs_u32(ptrs, lens, nr, None, None, ctypes.byref(tb), pp, None), "temp query")
+    temp = _temp(tb.value, out.device)
+    tb = ctypes.c_size_t(temp.numel())
+    with torch.cuda.device(out.device):
+        _check(L.bcf_merge_runs_ptrs_u32(ptrs, lens, nr, out.data_ptr(), temp.data_ptr(), ctypes.byref(tb), pp,
+                                         _stream(out)), "bcf_merge_runs_ptrs_u32")
+    return out[:n]
+
+
+def ipc_export(t) -> tuple:
+    """(handle bytes, byte offset of t's data in its allocation)."""
+    _require_cuda(t, "t")
+    h = ctypes.create_string_buffer(64)
+    off = ctypes.c_uint64(0)
+    _check(lib().bcf_ipc_export(t.data_ptr(), h, ctypes.byref(off)), "bcf_ipc_export")
+    return bytes(h.raw), int(off.value)
+
+
+def ipc_open(handle: bytes) -> int:
+    base = ctypes.c_void_p(0)
+    _check(lib().bcf_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(base)), "bcf_ipc_open")
+    return int(base.value)
+
+
+def ipc_close(base: int):
+    _check(lib().bcf_ipc_close(ctypes.c_void_p(base)), "bcf_ipc_close")
 
 
 SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}

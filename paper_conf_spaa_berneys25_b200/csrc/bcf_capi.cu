@@ -560,9 +560,13 @@ __global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __
     out[j] = __ldg(in + (n - 1 - j));
 }
 
-bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals, const uint64_t* h_run_offsets,
-                              int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals, void* d_temp,
-                              size_t* temp_bytes, const bcf_params* pp, void* stream) {
+// run_ptrs (host array of nruns device pointers, keys only): run r is read
+// from run_ptrs[r] (local or peer-mapped memory) instead of d_runs + offset;
+// pass 1 then reads every run through its own pointer (the plain kernel's
+// GroupDesc a_ptr / b_ptr), later passes are local
+static bcf_status merge_runs_impl(const uint32_t* d_runs, const uint32_t* const* run_ptrs, const uint32_t* d_run_vals,
+                                  const uint64_t* h_run_offsets, int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals,
+                                  void* d_temp, size_t* temp_bytes, const bcf_params* pp, void* stream) {
   // Pairwise merge tree over the runs in run order (run 2g is A, 2g+1 is B,
   // ties to A = the lower run).  Pass 1 reads the caller's ascending runs with
   // the plain table-mode kernel; it and every later non-final pass write odd
@@ -593,10 +597,13 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   }
   if (*temp_bytes < need) return BCF_ERROR_TEMP_TOO_SMALL;
   if (n == 0) return BCF_SUCCESS;
-  if (!d_runs || !d_out || (pairs && !d_out_vals)) return BCF_ERROR_INVALID_VALUE;
+  if ((!d_runs && !run_ptrs) || !d_out || (pairs && (!d_out_vals || run_ptrs))) return BCF_ERROR_INVALID_VALUE;
+  if (run_ptrs)
+    for (int r = 0; r < nruns; ++r)
+      if (!run_ptrs[r] && h_run_offsets[r + 1] > h_run_offsets[r]) return BCF_ERROR_INVALID_VALUE;
   cudaStream_t s = (cudaStream_t)stream;
   if (nruns == 1) {
-    cudaError_t e = cudaMemcpyAsync(d_out, d_runs, n * 4, cudaMemcpyDeviceToDevice, s);
+    cudaError_t e = cudaMemcpyAsync(d_out, run_ptrs ? run_ptrs[0] : d_runs, n * 4, cudaMemcpyDeviceToDevice, s);
     if (e == cudaSuccess && pairs) e = cudaMemcpyAsync(d_out_vals, d_run_vals, n * 4, cudaMemcpyDeviceToDevice, s);
     return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
   }
@@ -624,7 +631,7 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
   // (+8 B per B key), each at word phase A pos - len (mod 4) against its A
   // partner, read through src_kb / src_vb; A straight from the caller's
   // 16-byte aligned runs.  Bounded run count (one reverse launch per B run).
-  const bool rev1 = var.merge_win != nullptr && !tma_disabled() && nruns <= 64 &&
+  const bool rev1 = !run_ptrs && var.merge_win != nullptr && !tma_disabled() && nruns <= 64 &&
                     ((uintptr_t)d_runs & 15) == 0 &&
                     (!pairs || (((uintptr_t)d_run_vals & 15) == 0 &&
                                 (P > 1 || (((uintptr_t)d_out ^ (uintptr_t)d_out_vals) & 15) == 0)));
@@ -665,6 +672,12 @@ bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals
       gd.b_off = B.pos;
       gd.nb = B.len;
       gd.b_desc = B.desc;
+      if (i == 1 && run_ptrs) {  // the caller's runs, each through its own pointer
+        gd.a_ptr = run_ptrs[r];
+        gd.b_ptr = r + 1 < nr ? run_ptrs[r + 1] : run_ptrs[r];
+        gd.a_off = 0;
+        gd.b_off = 0;
+      }
       Run o{0, A.len + B.len, 0};
       if (!last) {
         o.desc = g & 1;
@@ -820,6 +833,68 @@ bcf_status bcf_set_op_u32(int32_t op, const uint32_t* d_a, uint64_t na, const ui
   e = launch("setop_compact", n, s, [&] {
     return setops::compact(op, M, V, (long long)n, counts, (unsigned long long*)d_count, d_out, d_out_src, s);
   });
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
+bcf_status bcf_merge_runs_u32(const uint32_t* d_runs, const uint32_t* d_run_vals, const uint64_t* h_run_offsets,
+                              int32_t nruns, uint32_t* d_out, uint32_t* d_out_vals, void* d_temp,
+                              size_t* temp_bytes, const bcf_params* pp, void* stream) {
+  return merge_runs_impl(d_runs, nullptr, d_run_vals, h_run_offsets, nruns, d_out, d_out_vals, d_temp, temp_bytes,
+                         pp, stream);
+}
+
+bcf_status bcf_merge_runs_ptrs_u32(const uint32_t* const* h_run_ptrs, const uint64_t* h_run_lens, int32_t nruns,
+                                   uint32_t* d_out, void* d_temp, size_t* temp_bytes, const bcf_params* pp,
+                                   void* stream) {
+  if (nruns < 0 || (nruns > 0 && (!h_run_ptrs || !h_run_lens))) return BCF_ERROR_INVALID_VALUE;
+  if (nruns > 4096) return BCF_ERROR_UNSUPPORTED;
+  uint64_t offs[4097];
+  offs[0] = 0;
+  for (int r = 0; r < nruns; ++r) offs[r + 1] = offs[r] + h_run_lens[r];
+  return merge_runs_impl(nullptr, d_temp ? h_run_ptrs : (const uint32_t* const*)nullptr, nullptr, offs, nruns, d_out,
+                         nullptr, d_temp, temp_bytes, pp, stream);
+}
+
+// ---- CUDA IPC (one node, one process per GPU; bcf_merge_runs_ptrs_u32) ----
+typedef int (*cuMemGetAddressRange_t)(unsigned long long*, size_t*, unsigned long long);
+static cuMemGetAddressRange_t address_range_fn() {
+  static cuMemGetAddressRange_t fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      f = nullptr;
+    return (cuMemGetAddressRange_t)f;
+  }();
+  return fn;
+}
+
+bcf_status bcf_ipc_export(const void* d_ptr, void* handle, uint64_t* offset) {
+  if (!d_ptr || !handle || !offset) return BCF_ERROR_INVALID_VALUE;
+  cuMemGetAddressRange_t range = address_range_fn();
+  if (!range) return BCF_ERROR_UNSUPPORTED;
+  unsigned long long base = 0;
+  size_t size = 0;
+  if (range(&base, &size, (unsigned long long)(uintptr_t)d_ptr) != 0) return BCF_ERROR_INVALID_VALUE;
+  cudaIpcMemHandle_t h;
+  cudaError_t e = cudaIpcGetMemHandle(&h, (void*)(uintptr_t)base);
+  if (e != cudaSuccess) return cuda_fail(e);
+  std::memcpy(handle, &h, sizeof(h));
+  *offset = (uint64_t)((uintptr_t)d_ptr - (uintptr_t)base);
+  return BCF_SUCCESS;
+}
+
+bcf_status bcf_ipc_open(const void* handle, void** d_base) {
+  if (!handle || !d_base) return BCF_ERROR_INVALID_VALUE;
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  cudaError_t e = cudaIpcOpenMemHandle(d_base, h, cudaIpcMemLazyEnablePeerAccess);
+  return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
+}
+
+bcf_status bcf_ipc_close(void* d_base) {
+  if (!d_base) return BCF_ERROR_INVALID_VALUE;
+  cudaError_t e = cudaIpcCloseMemHandle(d_base);
   return e == cudaSuccess ? BCF_SUCCESS : cuda_fail(e);
 }
 

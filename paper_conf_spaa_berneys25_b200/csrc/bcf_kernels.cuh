@@ -54,6 +54,10 @@ struct SortArgs {
 struct GroupDesc {
   long long a_off, na, b_off, nb, out_off, tile_begin;
   int a_desc, b_desc, out_desc, pad_;
+  // plain kernel, keys only: A / B keys read from these bases (any device or
+  // peer-mapped pointer, bcf_merge_runs_ptrs_u32) instead of src_k / src_kb
+  const uint32_t* a_ptr;
+  const uint32_t* b_ptr;
 };
 
 struct MergeArgs {
@@ -108,6 +112,9 @@ __device__ __forceinline__ GroupDesc group_of_tile(const MergeArgs& args, long l
     G.b_desc = args.cf_dirs;
     G.out_desc = args.cf_dirs && (g & 1);
     G.out_off = g0 + (G.out_desc ? ((2 * args.R - G.na - G.nb) & 3) : 0);
+    G.pad_ = 0;
+    G.a_ptr = nullptr;
+    G.b_ptr = nullptr;
   } else {
     int lo = 0, hi = args.ngroups - 1;  // last group with tile_begin <= tile
     while (lo < hi) {
@@ -419,8 +426,9 @@ __device__ __forceinline__ void merge_pass_tile(const MergeArgs& args, const lon
   long long j;
   const GroupDesc grp = group_of_tile(args, tile, T, j);
   const long long lenG = grp.na + grp.nb;
-  RunView Av{args.src_k + grp.a_off, grp.na, grp.a_desc};
-  const uint32_t* __restrict__ baseBk = args.src_kb ? args.src_kb : args.src_k;
+  const uint32_t* __restrict__ baseAk = grp.a_ptr ? grp.a_ptr : args.src_k;
+  const uint32_t* __restrict__ baseBk = grp.b_ptr ? grp.b_ptr : (args.src_kb ? args.src_kb : args.src_k);
+  RunView Av{baseAk + grp.a_off, grp.na, grp.a_desc};
   RunView Bv{baseBk + grp.b_off, grp.nb, grp.b_desc};
   const long long D0 = j * T;
   const long long D1 = D0 + T < lenG ? D0 + T : lenG;
@@ -452,7 +460,7 @@ __device__ __forceinline__ void merge_pass_tile(const MergeArgs& args, const lon
     const long long oA = grp.a_off + a0;
     const long long oB = CF ? (BDESC ? grp.b_off + grp.nb - b0 - T : grp.b_off + b0 + T - 1)
                             : grp.b_off + b0 - NA;
-    const uint32_t* __restrict__ pAk = args.src_k + oA;
+    const uint32_t* __restrict__ pAk = baseAk + oA;
     const uint32_t* __restrict__ pBk = baseBk + oB;
     const uint32_t* __restrict__ pAv = PAIRS ? args.src_v + oA : nullptr;
     const uint32_t* __restrict__ pBv = PAIRS ? (args.src_vb ? args.src_vb : args.src_v) + oB : nullptr;

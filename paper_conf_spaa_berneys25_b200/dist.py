@@ -200,11 +200,63 @@ class _PhaseMarks:
         return {n: self.ev[i].elapsed_time(self.ev[i + 1]) for i, n in enumerate(self.NAMES)}
 
 
-def sort(keys, values=None, group=None, ops=None, timing: list | None = None):
+class _PeerMaps:
+    """Peer allocations mapped into this process (CUDA IPC), by handle."""
+
+    def __init__(self):
+        self.maps = {}
+
+    def base(self, bcf, handle: bytes) -> int:
+        b = self.maps.get(handle)
+        if b is None:
+            b = bcf.ipc_open(handle)
+            self.maps[handle] = b
+        return b
+
+
+_PEERS = _PeerMaps()
+
+
+def _peer_exchange_merge(sk, send, group, ops, device):
+    """Fused exchange + merge: every rank exports the IPC
+    handle of its sorted shard, maps the others', and merges its p incoming
+    runs -- slice [cut_s(r), cut_s(r+1)) of rank s's shard, read in place over
+    NVLink -- with bcf_merge_runs_ptrs_u32, whose first pairwise pass reads the
+    peers' memory directly: no receive buffer, no separate copy."""
+    import torch
+    import torch.distributed as dist
+
+    bcf = ops.bcf
+    p = dist.get_world_size(group)
+    r = dist.get_rank(group)
+    cuts = np.concatenate([[0], np.cumsum(send)]).astype(np.int64)
+    handle, off = bcf.ipc_export(sk)
+    info = [None] * p
+    dist.all_gather_object(info, (handle, off, cuts.tolist()), group=group)
+    # every shard complete before anyone reads it
+    torch.cuda.current_stream(device).synchronize()
+    dist.barrier(group)
+    ptrs, lens = [], []
+    for s_ in range(p):
+        h, o, c = info[s_]
+        base = sk.data_ptr() - off if s_ == r else _PEERS.base(bcf, h)
+        ptrs.append(base + o + 4 * c[r])
+        lens.append(c[r + 1] - c[r])
+    out = bcf.merge_runs_ptrs(ptrs, lens, device, dtype=sk.dtype, params=ops.params)
+    # the peers have read this rank's shard before it can be reused
+    torch.cuda.current_stream(device).synchronize()
+    dist.barrier(group)
+    return out, lens
+
+
+def sort(keys, values=None, group=None, ops=None, timing: list | None = None, exchange: str = "nccl"):
     """Distributed stable sort of the shards held by the ranks of `group`.
     Returns (keys_out, values_out_or_None, DistStats).  keys: 1-D 4-byte
     tensor (u32 bit patterns in int32); values likewise.  `timing`: if a
-    list, a _PhaseMarks of this call is appended (CUDA tensors only)."""
+    list, a _PhaseMarks of this call is appended (CUDA tensors only).
+    exchange: "nccl" (all_to_all_single, then bcf_merge_runs_u32) or "peer"
+    (keys only, CUDA ops: the incoming runs are merged in place from the
+    peers' memory over CUDA IPC / NVLink by bcf_merge_runs_ptrs_u32)."""
     import torch
     import torch.distributed as dist
 
@@ -224,6 +276,18 @@ def sort(keys, values=None, group=None, ops=None, timing: list | None = None):
         return sk, sv, DistStats(0, [keys.numel()], [keys.numel()], [])
     marks.mark()
     send, pivots, rounds = exact_splitters(sk, sk.numel(), group, ops, device)
+    if exchange == "peer":
+        if values is not None or not isinstance(ops, CudaOps) or device.type != "cuda":
+            raise ValueError("exchange='peer' needs CUDA ops and keys only")
+        marks.mark()
+        ok, recv = _peer_exchange_merge(sk, send, group, ops, device)
+        marks.mark()
+        marks.mark()
+        if timing is not None:
+            timing.append(marks)
+        return ok, None, DistStats(rounds, send, recv, pivots)
+    elif exchange != "nccl":
+        raise ValueError(f"unknown exchange {exchange!r}")
     sc = torch.tensor(send, dtype=torch.int64, device=device)
     rc = torch.empty_like(sc)
     _all_to_all(rc, sc, group)

@@ -36,7 +36,7 @@ def _global_input(case):
     return si.uniform_u32(n_total, 4321) & np.uint32(mask), si.iota_u32(n_total)
 
 
-def _worker(rank, world, port, case, q):
+def _worker(rank, world, port, case, q, exchange="nccl"):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import paper_conf_spaa_berneys25_b200 as bcf
@@ -52,7 +52,7 @@ def _worker(rank, world, port, case, q):
         kt = torch.from_numpy(gk[lo:hi].view(np.int32).copy()).to(dev)
         vt = torch.from_numpy(gv[lo:hi].view(np.int32).copy()).to(dev) if with_vals else None
         launches0 = bcf.launch_count()
-        ok, ov, st = bdist.sort(kt, vt, ops=bdist.CudaOps())
+        ok, ov, st = bdist.sort(kt, vt, ops=bdist.CudaOps(), exchange=exchange)
         torch.cuda.synchronize()
         assert ok.is_cuda and bcf.launch_count() > launches0   # the library ran
         q.put((rank, ok.cpu().numpy().view(np.uint32).copy(),
@@ -64,17 +64,20 @@ def _worker(rank, world, port, case, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("case", [
-    (300001, 0xFFFFFFFF, True),    # distinct-ish keys, pairs, many tiles per rank
-    (200000, 0x7, True),           # 8 distinct keys: ties across the cut, stability
-    (123457, 0xFFFFFFFF, False),   # keys only, ragged
+@pytest.mark.parametrize("case,exchange", [
+    ((300001, 0xFFFFFFFF, True), "nccl"),    # distinct-ish keys, pairs, many tiles per rank
+    ((200000, 0x7, True), "nccl"),           # 8 distinct keys: ties across the cut, stability
+    ((123457, 0xFFFFFFFF, False), "nccl"),   # keys only, ragged
+    ((123457, 0xFFFFFFFF, False), "peer"),   # fused exchange + merge over CUDA IPC (f1)
+    ((400000, 0x3, False), "peer"),          # 4 distinct keys: ties across ranks, run order
+    ((3, 0xFF, False), "peer"),              # tiny: empty incoming runs
 ])
-def test_dist_sort_cuda_ops_world2_one_gpu(case):
+def test_dist_sort_cuda_ops_world2_one_gpu(case, exchange):
     world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q, exchange)) for r in range(world)]
     for p in procs:
         p.start()
     res = {}
