@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--u", type=int, default=0)
     ap.add_argument("--algo", type=int, default=0)
     ap.add_argument("--no-extras", action="store_true", help="skip e2e/cpu_baseline/contrast legs")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: all_to_all + run merge (nccl) or the fused peer-memory merge (peer)")
     return ap.parse_args()
 
 
@@ -204,6 +206,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         ("pairs_u32_2^26", 1 << 26, 16),
         ("merge_u32_2x2^25", 1 << 26, 8),
         ("merge_runs_8x2^23", 1 << 26, 24),  # 3 pairwise passes x 8 B/key
+        ("set_intersection_2x2^25", 1 << 26, 8),
     ]
     for name, n, bpk in legs:
         if name.startswith("f32"):
@@ -211,6 +214,15 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             out = torch.empty_like(x)
             run = lambda: bcf.sort(x, out=out, params=params, temp=temp)  # noqa: E731
             workload = "2^28 float32 keys, uniform [0,1) (24-bit mantissa grid), IEEE totalOrder"
+        elif name.startswith("set_"):
+            # bcf_set_op_u32: intersection of two sorted
+            # 2^25 arrays drawn from 2^26 values (about half the keys common)
+            prm = params
+            sa_ = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(7), dev) & 0x3FFFFFF, params=prm)
+            sb_ = bcf.sort(si.uniform_u32_torch(n // 2, si.config_seed(7), dev, lo=n // 2) & 0x3FFFFFF, params=prm)
+            run = lambda: bcf.set_op("intersection", sa_, sb_, params=prm)  # noqa: E731
+            workload = ("bcf_set_op_u32 intersection of two sorted 2^25 uint32 arrays over 2^26 values "
+                        "(tags, CF merge with tags, keep flags, compaction; includes the count read-back)")
         elif name.startswith("merge_runs"):
             # bcf_merge_runs_u32: the distributed sort's final local merge at p = 8
             prm = params
@@ -236,7 +248,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
             prm = bcf.default_pairs_params()  # pairs default (11, 256)
             run = lambda: bcf.sort_pairs(k, v, ko, vo, params=prm, temp=temp)  # noqa: E731
             workload = "2^26 uint32 (key & 0xFFFF, heavy duplicates) + uint32 value (index) pairs, stable"
-        if name.startswith("f32") or name.startswith("merge"):
+        if name.startswith(("f32", "merge", "set_")):
             prm = params
         temp = bcf.temp_buffer(n, prm, pairs=name.startswith("pairs"), device=dev)
         for _ in range(3):
@@ -257,7 +269,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
         torch.cuda.synchronize()
         bcf.profile_enable(False)
         prof = bcf.profile_collect()
-        cls = "merge_runs" if name.startswith("merge_runs") else ("merge" if name.startswith("merge") else
+        cls = "merge_runs" if name.startswith("merge_runs") else ("merge" if name.startswith(("merge", "set_")) else
                                                                    ("merge_passes" if "merge_passes" in prof
                                                                     else "merge_pass"))
         mp = prof.get(cls, {"launches": 0, "total_ms": 0.0, "keys": 0})
@@ -276,7 +288,7 @@ def extra_configs(bcf, dev, stream, flush, params, peaks, steps=10):
                                     "frac_of_hbm": (bpl / (avg / 1e3) / 1e9) / peaks["hbm_gbs"] if avg else None,
                                     "bytes_per_launch": bpl, "passes_per_launch": bpl / (bpk * n)},
                      # merge legs: algorithmic bytes of the whole call / call time
-                     "call_gbs_algorithmic": bpk * n / (ms / 1e3) / 1e9 if name.startswith("merge") else None,
+                     "call_gbs_algorithmic": bpk * n / (ms / 1e3) / 1e9 if name.startswith(("merge", "set_")) else None,
                      "block_sort_ms": bs["total_ms"] / max(1, bs["launches"])}
         del run, temp
         torch.cuda.empty_cache()
@@ -405,7 +417,7 @@ def main():
         x = inputs[i % 2] if x is None else x
         if world == 1:
             return bcf.sort(x, out=out, params=params, temp=temp)
-        ko, _, st = bdist.sort(x, ops=bdist.CudaOps(params), timing=timing)
+        ko, _, st = bdist.sort(x, ops=bdist.CudaOps(params), timing=timing, exchange=a.exchange)
         if timing is not None:
             dist_sends.append(st.send_counts)
         return ko
@@ -526,6 +538,28 @@ def main():
         "clocks": clk.summary(),
     }
     if distributed is not None:
+        distributed["exchange_mode"] = a.exchange
+        if a.exchange == "nccl":
+            # context: the fused exchange + merge over peer memory on
+            # the same inputs, timed the same way (max over ranks)
+            try:
+                kp = min(a.steps, 10)
+                for i in range(2):
+                    bdist.sort(inputs[i % 2], ops=bdist.CudaOps(params), exchange="peer")
+                pev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(kp)]
+                dist.barrier()
+                torch.cuda.synchronize()
+                for i in range(kp):
+                    flush.fill_(i)
+                    pev[i][0].record(stream)
+                    bdist.sort(inputs[i % 2], ops=bdist.CudaOps(params), exchange="peer")
+                    pev[i][1].record(stream)
+                torch.cuda.synchronize()
+                pt = torch.tensor([sum(s_.elapsed_time(e_) for s_, e_ in pev)], dtype=torch.float64, device=dev)
+                dist.all_reduce(pt, op=dist.ReduceOp.MAX)
+                distributed["peer_exchange_keys_per_s"] = kp * n_total / (float(pt.item()) / 1e3)
+            except Exception as ex:  # noqa: BLE001
+                distributed["peer_exchange_error"] = repr(ex)[:200]
         line["distributed"] = distributed
 
     # ---- e2e through the public API, host buffers, copies inside the region
