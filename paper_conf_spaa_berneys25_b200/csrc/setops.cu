@@ -113,17 +113,24 @@ __device__ __forceinline__ bool keep(int op, const uint32_t* __restrict__ M, con
   return (op == 0 || op == 3) && k >= m;
 }
 
+// keep bits of a block's BLK merged positions, striped: bit q of thread t is
+// position base + q * THREADS + t (every load of a row is coalesced)
+__device__ __forceinline__ uint32_t keep_bits(int op, const uint32_t* __restrict__ M, const uint32_t* __restrict__ V,
+                                              long long n, long long base) {
+  uint32_t mask = 0;
+#pragma unroll 4
+  for (int q = 0; q < ITEMS; ++q) {
+    const long long p = base + (long long)q * THREADS + threadIdx.x;
+    if (p < n && keep(op, M, V, n, p)) mask |= 1u << q;
+  }
+  return mask;
+}
+
 // per-block keep counts
 __global__ void __launch_bounds__(THREADS) count_kernel(int op, const uint32_t* __restrict__ M,
                                                         const uint32_t* __restrict__ V, long long n,
                                                         unsigned long long* __restrict__ counts) {
-  const long long base = blockIdx.x * BLK + (long long)threadIdx.x * ITEMS;
-  int c = 0;
-#pragma unroll 4
-  for (int q = 0; q < ITEMS; ++q) {
-    const long long p = base + q;
-    if (p < n && keep(op, M, V, n, p)) ++c;
-  }
+  int c = __popc(keep_bits(op, M, V, n, blockIdx.x * BLK));
   for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
   __shared__ int ws[THREADS / 32];
   if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
@@ -165,33 +172,38 @@ __global__ void __launch_bounds__(THREADS) scatter_kernel(int op, const uint32_t
                                                           const uint32_t* __restrict__ V, long long n,
                                                           const unsigned long long* __restrict__ offsets,
                                                           uint32_t* __restrict__ out, uint32_t* __restrict__ out_src) {
-  const long long base = blockIdx.x * BLK + (long long)threadIdx.x * ITEMS;
-  uint32_t mask = 0;
-#pragma unroll 4
-  for (int q = 0; q < ITEMS; ++q) {
-    const long long p = base + q;
-    if (p < n && keep(op, M, V, n, p)) mask |= 1u << q;
-  }
-  const int c = __popc(mask);
-  // block-wide exclusive scan of c
+  constexpr int NWARP = THREADS / 32;
+  const long long base = blockIdx.x * BLK;
+  const uint32_t mask = keep_bits(op, M, V, n, base);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  int inc = c;
-  for (int o = 1; o < 32; o <<= 1) {
-    const int v = __shfl_up_sync(0xffffffffu, inc, o);
-    if (lane >= o) inc += v;
-  }
-  __shared__ int ws[THREADS / 32];
-  if (lane == 31) ws[warp] = inc;
-  __syncthreads();
-  int wbase = 0;
-  for (int w = 0; w < warp; ++w) wbase += ws[w];
-  unsigned long long o = offsets[blockIdx.x] + (unsigned long long)(wbase + inc - c);
+  // kept count of every (row q, warp w) segment, then their exclusive scan in
+  // merged order (row-major: position base + q THREADS + 32 w + lane)
+  __shared__ int seg[ITEMS * NWARP];
+  uint32_t bal[ITEMS];
+#pragma unroll
   for (int q = 0; q < ITEMS; ++q) {
-    if (mask & (1u << q)) {
-      const long long p = base + q;
+    bal[q] = __ballot_sync(0xffffffffu, (mask >> q) & 1u);
+    if (lane == 0) seg[q * NWARP + warp] = __popc(bal[q]);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int k = 0; k < ITEMS * NWARP; ++k) {
+      const int c = seg[k];
+      seg[k] = run;
+      run += c;
+    }
+  }
+  __syncthreads();
+  const unsigned long long o0 = offsets[blockIdx.x];
+  const uint32_t lt = (1u << lane) - 1u;
+#pragma unroll
+  for (int q = 0; q < ITEMS; ++q) {
+    if ((mask >> q) & 1u) {
+      const long long p = base + (long long)q * THREADS + threadIdx.x;
+      const unsigned long long o = o0 + (unsigned long long)(seg[q * NWARP + warp] + __popc(bal[q] & lt));
       out[o] = __ldg(M + p);
       if (out_src) out_src[o] = __ldg(V + p);
-      ++o;
     }
   }
 }
