@@ -25,6 +25,13 @@
 
 namespace bcf {
 
+// L2 hints of the window kernel's bulk copies (A/B builds): bit 0 = window
+// loads evict_first (the pass's input is dead once read), bit 1 = output
+// stores evict_last (the next pass reads them)
+#ifndef BCF_L2_HINTS
+#define BCF_L2_HINTS 0
+#endif
+
 #ifndef BCF_WIN_Q
 #define BCF_WIN_Q 1  // span S2 = T + Q * T/4 (Q = 4: two full windows, never exhausted)
 #endif
@@ -335,8 +342,15 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       }
       if (lane == 0) {
         tma::mbar_expect_tx(&full_bar[s], (uint32_t)(a_hi + (b_hi - b_lo)) * 4u * (PAIRS ? 2u : 1u));
-        if (a_hi > 0) tma::bulk_g2s(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
-        if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, srcB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        if constexpr ((BCF_L2_HINTS & 1) != 0) {
+          const uint64_t pol = tma::policy_evict_first();
+          if (a_hi > 0) tma::bulk_g2s_hint(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s], pol);
+          if (b_hi > b_lo)
+            tma::bulk_g2s_hint(sk + b_lo, srcB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s], pol);
+        } else {
+          if (a_hi > 0) tma::bulk_g2s(sk, src + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
+          if (b_hi > b_lo) tma::bulk_g2s(sk + b_lo, srcB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+        }
         if constexpr (PAIRS) {
           uint32_t* sv = stage_v(s);
           if (a_hi > 0) tma::bulk_g2s(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
@@ -390,7 +404,11 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       int ilo = align_up4(w0), ihi = align_dn4(w1);
       if (lane == 0) {
         if (ihi > ilo) {
-          tma::bulk_s2g(args.dst_k + (M.c0 - M.cout) + ilo, stage(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
+          if constexpr ((BCF_L2_HINTS & 2) != 0)
+            tma::bulk_s2g_hint(args.dst_k + (M.c0 - M.cout) + ilo, stage(s) + ilo, (uint32_t)(ihi - ilo) * 4u,
+                               tma::policy_evict_last());
+          else
+            tma::bulk_s2g(args.dst_k + (M.c0 - M.cout) + ilo, stage(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
           if constexpr (PAIRS)
             tma::bulk_s2g(args.dst_v + (M.c0 - M.cout) + ilo, stage_v(s) + ilo, (uint32_t)(ihi - ilo) * 4u);
         }
