@@ -15,8 +15,8 @@
 //      run bounds by exponential + binary search around each position (one
 //      or two loads for short runs), the A/B boundary of a run by binary
 //      search on the tags;
-//   4. compaction: per-block keep counts, one-block exclusive scan, scatter
-//      of the kept keys (and their tags) in merged order.
+//   4. compaction in one pass (decoupled look-back over per-block keep
+//      counts), scatter of the kept keys (and their tags) in merged order.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -126,59 +126,40 @@ __device__ __forceinline__ uint32_t keep_bits(int op, const uint32_t* __restrict
   return mask;
 }
 
-// per-block keep counts
-__global__ void __launch_bounds__(THREADS) count_kernel(int op, const uint32_t* __restrict__ M,
-                                                        const uint32_t* __restrict__ V, long long n,
-                                                        unsigned long long* __restrict__ counts) {
-  int c = __popc(keep_bits(op, M, V, n, blockIdx.x * BLK));
-  for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
-  __shared__ int ws[THREADS / 32];
-  if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    int t = 0;
-    for (int w = 0; w < THREADS / 32; ++w) t += ws[w];
-    counts[blockIdx.x] = (unsigned long long)t;
-  }
+// single-pass compaction (decoupled look-back): blocks take tiles in order
+// from a counter, publish their keep count (AGGREGATE) at once, then walk
+// back over their predecessors' words until an inclusive PREFIX, publish
+// their own PREFIX and scatter.  status[b] = flag << 62 | value (0 = not
+// ready); the last tile writes the total.
+constexpr unsigned long long ST_AGG = 1ull << 62, ST_PRE = 2ull << 62, ST_VAL = (1ull << 62) - 1;
+
+__device__ __forceinline__ unsigned long long ld_acq(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_rel(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// exclusive scan of nb block counts in place (one CTA); total -> *total
-__global__ void __launch_bounds__(1024) scan_kernel(unsigned long long* __restrict__ counts, long long nb,
-                                                    unsigned long long* __restrict__ total) {
-  const int t = threadIdx.x;
-  const long long per = (nb + 1023) / 1024;
-  const long long b0 = t * per, b1 = b0 + per < nb ? b0 + per : nb;
-  unsigned long long s = 0;
-  for (long long b = b0; b < b1; ++b) s += counts[b];
-  __shared__ unsigned long long sh[1024];
-  sh[t] = s;
-  __syncthreads();
-  for (int o = 1; o < 1024; o <<= 1) {  // inclusive Hillis-Steele scan
-    const unsigned long long v = t >= o ? sh[t - o] : 0ull;
-    __syncthreads();
-    sh[t] += v;
-    __syncthreads();
-  }
-  unsigned long long run = t ? sh[t - 1] : 0ull;
-  for (long long b = b0; b < b1; ++b) {
-    const unsigned long long c = counts[b];
-    counts[b] = run;
-    run += c;
-  }
-  if (t == 1023) *total = sh[1023];
-}
-
-__global__ void __launch_bounds__(THREADS) scatter_kernel(int op, const uint32_t* __restrict__ M,
-                                                          const uint32_t* __restrict__ V, long long n,
-                                                          const unsigned long long* __restrict__ offsets,
-                                                          uint32_t* __restrict__ out, uint32_t* __restrict__ out_src) {
+__global__ void __launch_bounds__(THREADS) compact_lookback_kernel(int op, const uint32_t* __restrict__ M,
+                                                                   const uint32_t* __restrict__ V, long long n,
+                                                                   unsigned long long* __restrict__ status,
+                                                                   unsigned int* __restrict__ ticket,
+                                                                   unsigned long long* __restrict__ total,
+                                                                   uint32_t* __restrict__ out,
+                                                                   uint32_t* __restrict__ out_src) {
   constexpr int NWARP = THREADS / 32;
-  const long long base = blockIdx.x * BLK;
+  __shared__ long long s_tile;
+  __shared__ int seg[ITEMS * NWARP];
+  __shared__ unsigned long long s_excl;
+  if (threadIdx.x == 0) s_tile = atomicAdd(ticket, 1u);
+  __syncthreads();
+  const long long b = s_tile;
+  const long long nb = (n + BLK - 1) / BLK;
+  const long long base = b * BLK;
   const uint32_t mask = keep_bits(op, M, V, n, base);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  // kept count of every (row q, warp w) segment, then their exclusive scan in
-  // merged order (row-major: position base + q THREADS + 32 w + lane)
-  __shared__ int seg[ITEMS * NWARP];
   uint32_t bal[ITEMS];
 #pragma unroll
   for (int q = 0; q < ITEMS; ++q) {
@@ -186,16 +167,57 @@ __global__ void __launch_bounds__(THREADS) scatter_kernel(int op, const uint32_t
     if (lane == 0) seg[q * NWARP + warp] = __popc(bal[q]);
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int run = 0;
-    for (int k = 0; k < ITEMS * NWARP; ++k) {
-      const int c = seg[k];
-      seg[k] = run;
-      run += c;
+  if (warp == 0) {
+    // exclusive scan of the ITEMS * NWARP segment counts (4 per lane)
+    int v[ITEMS * NWARP / 32];
+    int sum = 0;
+#pragma unroll
+    for (int k = 0; k < ITEMS * NWARP / 32; ++k) {
+      v[k] = seg[lane * (ITEMS * NWARP / 32) + k];
+      sum += v[k];
+    }
+    int inc = sum;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += t;
+    }
+    int run = inc - sum;
+#pragma unroll
+    for (int k = 0; k < ITEMS * NWARP / 32; ++k) {
+      seg[lane * (ITEMS * NWARP / 32) + k] = run;
+      run += v[k];
+    }
+    const unsigned long long cnt = (unsigned long long)__shfl_sync(0xffffffffu, inc, 31);
+    // publish, then look back
+    unsigned long long excl = 0;
+    if (b == 0) {
+      if (lane == 0) st_rel(status, ST_PRE | cnt);
+    } else {
+      if (lane == 0) st_rel(status + b, ST_AGG | cnt);
+      long long k0 = b - 1;  // window [k0 - 31, k0]
+      while (true) {
+        const long long k = k0 - lane;
+        unsigned long long w = k >= 0 ? ld_acq(status + k) : ST_PRE;  // before tile 0: prefix 0
+        const unsigned ready = __ballot_sync(0xffffffffu, w != 0ull);
+        const unsigned pre = __ballot_sync(0xffffffffu, (w & ~ST_VAL) == ST_PRE);
+        const int first_pre = pre ? __ffs(pre) - 1 : 32;  // nearest prefix in the window
+        const unsigned need = first_pre < 31 ? ((2u << first_pre) - 1u) : 0xffffffffu;
+        if ((ready & need) != need) continue;  // a predecessor not yet published: re-read
+        unsigned long long add = (lane <= first_pre && k >= 0) ? (w & ST_VAL) : 0ull;
+        for (int o = 16; o > 0; o >>= 1) add += __shfl_xor_sync(0xffffffffu, add, o);
+        excl += add;
+        if (first_pre < 32) break;
+        k0 -= 32;
+      }
+      if (lane == 0) st_rel(status + b, ST_PRE | (excl + cnt));
+    }
+    if (lane == 0) {
+      s_excl = excl;
+      if (b == nb - 1) *total = excl + cnt;
     }
   }
   __syncthreads();
-  const unsigned long long o0 = offsets[blockIdx.x];
+  const unsigned long long o0 = s_excl;
   const uint32_t lt = (1u << lane) - 1u;
 #pragma unroll
   for (int q = 0; q < ITEMS; ++q) {
@@ -210,13 +232,15 @@ __global__ void __launch_bounds__(THREADS) scatter_kernel(int op, const uint32_t
 
 // launches 3 and 4 (the flags, scan and scatter kernels); M, V merged keys
 // and tags of n elements; counts: nblocks + 1 words of temp
+// counts: nblocks + 1 words of temp (look-back status words + the ticket)
 cudaError_t compact(int op, const uint32_t* M, const uint32_t* V, long long n, unsigned long long* counts,
                     unsigned long long* d_count, uint32_t* out, uint32_t* out_src, cudaStream_t s) {
   const long long nb = (n + BLK - 1) / BLK;
   if (nb == 0) return cudaMemsetAsync(d_count, 0, sizeof(unsigned long long), s);
-  count_kernel<<<(unsigned)nb, THREADS, 0, s>>>(op, M, V, n, counts);
-  scan_kernel<<<1, 1024, 0, s>>>(counts, nb, d_count);
-  scatter_kernel<<<(unsigned)nb, THREADS, 0, s>>>(op, M, V, n, counts, out, out_src);
+  cudaError_t e = cudaMemsetAsync(counts, 0, (size_t)(nb + 1) * sizeof(unsigned long long), s);
+  if (e != cudaSuccess) return e;
+  compact_lookback_kernel<<<(unsigned)nb, THREADS, 0, s>>>(op, M, V, n, counts, (unsigned int*)(counts + nb),
+                                                           d_count, out, out_src);
   return cudaGetLastError();
 }
 
