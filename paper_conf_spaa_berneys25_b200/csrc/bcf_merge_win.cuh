@@ -92,6 +92,42 @@ __device__ __forceinline__ int warp_prefix_count(int n, P pred, int lane) {
   return lo;
 }
 
+// The same count for a window stored through rho (E sharing factors with w):
+// key(m) reads logical word l0 + sgn * m.  Probes at stride f E (f odd) form a
+// round set (Lemma 1 / Cor. 3), so every round reads 32 distinct banks; the
+// last <= E candidates are consecutive words, read in two halves split at the
+// rho partition boundary (consecutive words inside one partition are
+// consecutive banks modulo its rotation).
+template <int E, class P>
+__device__ __forceinline__ int warp_prefix_count_rho(int n, P pred, int l0, int sgn, int lane) {
+  int lo = 0, hi = n;
+  while (hi - lo > E) {
+    const int need = ((hi - lo) + 31) >> 5;
+    const int f = ((need + E - 1) / E) | 1;
+    const int st = f * E;
+    const int m = lo + (lane + 1) * st - 1;
+    const bool p = m < hi && pred(m);
+    const int c = __popc(__ballot_sync(FULL, p));
+    const int nlo = lo + c * st;
+    int nhi = lo + (c + 1) * st - 1;
+    if (nhi > hi) nhi = hi;
+    lo = nlo;
+    hi = nhi;
+  }
+  const int m = lo + lane;
+  const bool act = m < hi;
+  // logical word of candidate m, and the partition boundary after lo's word
+  const int w0 = l0 + sgn * lo;
+  const int pend = sgn > 0 ? rho_partition_end<E>(w0) : rho_partition_end<E>(w0) - W * E / cgcd(W, E);
+  const int wm = l0 + sgn * m;
+  const bool first = sgn > 0 ? wm < pend : wm >= pend;
+  bool p = false;
+  if (act && first) p = pred(m);
+  __syncwarp();
+  if (act && !first) p = pred(m);
+  return lo + __popc(__ballot_sync(FULL, p));
+}
+
 // resident CTAs per SM the kernel is built for (5 at u = 128)
 template <int U, bool PAIRS = false>
 __host__ __device__ constexpr int win_min_blocks() {
@@ -283,19 +319,19 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         if (pb1 > pb0) tma::bulk_prefetch_l2(srcB + pb0, (uint32_t)(pb1 - pb0) * 4u);
       };
       if constexpr (RHO) {
-        // logical word q of the window at physical slot rho(q): A from
-        // src[oA + q] (q < WA), B from srcB[oB + q] (q >= S2 - WB); one
-        // warp-wide 4-byte cp.async per 32 consecutive words (coalesced
-        // reads, rotated conflict-free writes)
+        // staged in PHYSICAL order: slot p (32 consecutive slots per warp
+        // instruction, conflict-free writes) receives logical word
+        // q = rho^-1(p): A from src[oA + q] (q < WA), B from srcB[oB + q]
+        // (q >= S2 - WB = WA); the reads stay inside one or two rotated
+        // partitions (coalesced)
         __syncwarp();  // meta[s] written before any lane's copies land
         uint32_t* sk = stage(s);
-        for (int q = lane; q < WA; q += W) {
-          tma::cp_async4(sk + rho<E>(q), src + oA + q);
-          if constexpr (PAIRS) tma::cp_async4(stage_v(s) + rho<E>(q), srcv + oA + q);
-        }
-        for (int q = S2 - WB + lane; q < S2; q += W) {
-          tma::cp_async4(sk + rho<E>(q), srcB + oB + q);
-          if constexpr (PAIRS) tma::cp_async4(stage_v(s) + rho<E>(q), srcvB + oB + q);
+        for (int p = lane; p < S2; p += W) {
+          const int q = rho_inv<E>(p);
+          if (q >= WA && q < S2 - WB) continue;  // the gap between the windows (never read)
+          const uint32_t* g = q < WA ? src + oA + q : srcB + oB + q;
+          tma::cp_async4(sk + p, g);
+          if constexpr (PAIRS) tma::cp_async4(stage_v(s) + p, (q < WA ? srcv + oA : srcvB + oB) + q);
         }
         if (lane == 0) {
           prefetch_next();
@@ -527,12 +563,20 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
       if (!(M.fin & 1) && r == WA) {
         // A window exhausted at D_A = WA + #{B[y] < A[WA-1]} (ties go to A)
         const uint32_t v = lds<E>(sk, WA - 1);
-        const int nb = warp_prefix_count(WB, [&](int y) { return lds<E>(sk, S2 - 1 - y) < v; }, lane);
+        int nb;
+        if constexpr (RHO)
+          nb = warp_prefix_count_rho<E>(WB, [&](int y) { return lds<E>(sk, S2 - 1 - y) < v; }, S2 - 1, -1, lane);
+        else
+          nb = warp_prefix_count(WB, [&](int y) { return sk[S2 - 1 - y] < v; }, lane);
         cnt = WA + nb;
       } else if (!(M.fin & 2) && cmax - r == WB) {
         // B window exhausted at D_B = WB + #{A[x] <= B[WB-1]}
         const uint32_t v = lds<E>(sk, S2 - WB);
-        const int na = warp_prefix_count(WA, [&](int x) { return !(v < lds<E>(sk, x)); }, lane);
+        int na;
+        if constexpr (RHO)
+          na = warp_prefix_count_rho<E>(WA, [&](int x) { return !(v < lds<E>(sk, x)); }, 0, 1, lane);
+        else
+          na = warp_prefix_count(WA, [&](int x) { return !(v < sk[x]); }, lane);
         cnt = WB + na;
       }
       if (cnt < cmax) {
