@@ -394,9 +394,16 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
         }
         if constexpr (PAIRS) {
           uint32_t* sv = stage_v(s);
-          if (a_hi > 0) tma::bulk_g2s(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
-          if (b_hi > b_lo)
-            tma::bulk_g2s(sv + b_lo, srcvB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+          if constexpr ((BCF_L2_HINTS & 1) != 0) {
+            const uint64_t pol = tma::policy_evict_first();
+            if (a_hi > 0) tma::bulk_g2s_hint(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s], pol);
+            if (b_hi > b_lo)
+              tma::bulk_g2s_hint(sv + b_lo, srcvB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s], pol);
+          } else {
+            if (a_hi > 0) tma::bulk_g2s(sv, srcv + (oA - c), (uint32_t)a_hi * 4u, &full_bar[s]);
+            if (b_hi > b_lo)
+              tma::bulk_g2s(sv + b_lo, srcvB + (oB + b_lo - c), (uint32_t)(b_hi - b_lo) * 4u, &full_bar[s]);
+          }
         }
         prefetch_next();
       }
