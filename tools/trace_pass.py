@@ -12,6 +12,8 @@ buf = np.zeros(1 << 21, dtype=np.uint64)
 bcf.lib().bcf_debug_trace_copy.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
 assert bcf.lib().bcf_debug_trace_copy(buf.ctypes.data, buf.nbytes) == 0
 tr = buf.reshape(-1, 256).astype(np.int64)
+if os.environ.get("TRACE_SAVE"):
+    np.savez_compressed(os.environ["TRACE_SAVE"], tr=tr[np.nonzero(tr[:, 0])[0]])
 ctas = np.nonzero(tr[:, 0])[0]
 t0 = tr[ctas, 0].min()
 print("ctas", len(ctas), "kernel span us %.1f" % ((tr[ctas].max() - t0) / 1e3))
