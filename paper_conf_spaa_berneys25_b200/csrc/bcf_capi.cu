@@ -146,6 +146,21 @@ static int bs_threads(const Params& p, bool cf, bool pairs) {
   return p.U;
 }
 
+// Two-tile block sort (keys-only CF at E = 31, block tiles of 256 threads):
+// runs of 2 x 7936 keys, one merge pass fewer.  Opt-in, BCF_BS2=1
+// (read per call): measured slower at 2^24, the extra shared-memory level
+// costs 35 us against the 30 us merge pass it saves
+// (profiles/r02_ab_block_sort2_2p24.txt).
+static bool bs2_enabled() {
+  const char* v = getenv("BCF_BS2");
+  return v && v[0] == '1';
+}
+static bool use_bs2(const Params& p, bool cf, bool pairs, int Ubs) {
+  if (!cf || pairs || !bs2_enabled() || Ubs != 256) return false;
+  const Variant& v = launch_table().v[p.E][u_index(Ubs)][0][0];
+  return v.block_sort2 != nullptr;
+}
+
 // BCF_TRACE=<pass>: record a per-CTA timeline of that merge pass (debug)
 static unsigned long long* g_trace = nullptr;
 static const size_t TRACE_WORDS = 1 << 21;
@@ -261,12 +276,14 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   const int Ubs = bs_threads(p, cf, pairs);
   const Variant& vbs = launch_table().v[p.E][u_index(Ubs)][p.algo][pairs ? 1 : 0];
   if (!vbs.block_sort) return BCF_ERROR_UNSUPPORTED;
+  const bool one_sm = one_cta_per_sm();
+  const bool bs2 = !one_sm && use_bs2(p, cf, pairs, Ubs);
   const long long T = (long long)p.U * p.E;
-  const long long Tbs = (long long)Ubs * p.E;
+  const long long Tbs = (long long)Ubs * p.E * (bs2 ? 2 : 1);  // the block sort's run length
   const long long tiles = (long long)((n + T - 1) / T);
   const long long tiles_bs = (long long)((n + Tbs - 1) / Tbs);
-  int lg_bs = 0;
-  while ((p.U << lg_bs) < Ubs) ++lg_bs;
+  int lg_bs = 0;  // log2(Tbs / T)
+  while ((T << lg_bs) < Tbs) ++lg_bs;
   int P = 0;
   while ((Tbs << P) < (long long)n) ++P;
   const bool use_tma = cf && var.merge_tma != nullptr && !tma_disabled();
@@ -289,13 +306,14 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   // the block sort zeroes the progress flags (no memset between the two launches)
   SortArgs sa{in_k, in_v, P == 0 ? out_k : X, P == 0 ? out_v : XV, (long long)n, f32 ? 1 : 0,
               (f32 && P == 0) ? 1 : 0, cf ? 1 : 0, multi ? progress : nullptr, multi ? MAX_PROGRESS_CTAS : 0};
-  const bool one_sm = one_cta_per_sm();
   long long grid_bs = tiles_bs;
   if (one_sm && tiles_bs > sm_count()) {
     grid_bs = sm_count();
     sa.ntiles = tiles_bs;
   }
-  cudaError_t e = launch("block_sort", n, s, [&] { return vbs.block_sort(sa, grid_bs, s); });
+  cudaError_t e = launch("block_sort", n, s, [&] {
+    return bs2 ? vbs.block_sort2(sa, grid_bs, s) : vbs.block_sort(sa, grid_bs, s);
+  });
   if (e != cudaSuccess) return cuda_fail(e);
   if (multi) {
     MergeArgs ma{X, XV, out_k, out_v, (long long)n, Tbs, 1 + lg_bs, f32 ? 1 : 0, cf ? 1 : 0, nullptr, 0, nullptr};
@@ -486,7 +504,8 @@ bcf_status bcf_sort_plan(uint64_t n, const bcf_params* pp, int32_t pairs, int64_
   bcf_status st = resolve(pp, p, pairs != 0);
   if (st != BCF_SUCCESS) return st;
   const bool cf = p.algo == BCF_ALGO_CONFLICT_FREE;
-  const long long Tbs = (long long)bs_threads(p, cf, pairs != 0) * p.E;
+  const int Ubs = bs_threads(p, cf, pairs != 0);
+  const long long Tbs = (long long)Ubs * p.E * (!one_cta_per_sm() && use_bs2(p, cf, pairs != 0, Ubs) ? 2 : 1);
   int P = 0;
   while ((Tbs << P) < (long long)n) ++P;
   if (block_sort_tile) *block_sort_tile = Tbs;

@@ -199,24 +199,20 @@ __host__ __device__ constexpr int bs_min_blocks() {
   return U == 256 ? BCF_BS_MINB256 : (U == 512 ? BCF_BS_MINB512 : 0);
 }
 
+// The block sort of one tile of T = U*E keys (input t0 .. t0+cnt of
+// args.in_k, pads = max key): on return, thread tid holds the sorted tile's
+// outputs [tid E, tid E + E) in key[] (val[] for pairs); sk / sv (tile_words
+// each) are its working buffers, still being read by other threads until the
+// caller's next __syncthreads.
 template <int E, int U, bool PAIRS, bool CF>
-__device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long long tile) {
-  constexpr int T = U * E;
+__device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* sk, uint32_t* sv,
+                                                const long long t0, const int cnt, uint32_t (&key)[E],
+                                                uint32_t (&val)[E]) {
   constexpr int NW = U / W;
-  extern __shared__ __align__(16) uint32_t smem_dyn[];
-  uint32_t* sk = smem_dyn;                      // tile_words keys
-  uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
   __shared__ int s_org[NW + 1];
   const int tid = threadIdx.x;
   const int lane = tid & (W - 1);
   const int warp = tid >> 5;
-  const long long t0 = tile * T;
-  const long long rem = args.n - t0;
-  const int cnt = rem < T ? (int)rem : T;
-  tma::pdl_wait();  // the input may be produced by the preceding grid
-  // (after the wait: the preceding grid may be a merge launch using the flags)
-  if (args.zero != nullptr && tile == 0)
-    for (int k = tid; k < args.nzero; k += U) args.zero[k] = 0u;
 
   // keys only, E = 31: levels 0..4 (runs up to one warp) run in registers
   // across the warp (warp_bitonic_levels); any assignment of the warp's 992
@@ -224,7 +220,7 @@ __device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long
   // memory (coalesced: key r of lane l is element 32 r + l of the warp's
   // chunk) without the shared-memory round trip of the general path
   constexpr bool WARP_PHASE = CF && !PAIRS && E + 1 == W && U >= 2 * W;
-  uint32_t key[E], val[E], tag[E];
+  uint32_t tag[E];
   if constexpr (WARP_PHASE) {
     const int wbase = warp * (W * E);
     const uint32_t* __restrict__ gin_k = args.in_k + t0 + wbase + lane;
@@ -387,6 +383,24 @@ __device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long
       }
     }
   }
+}
+
+template <int E, int U, bool PAIRS, bool CF>
+__device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long long tile) {
+  constexpr int T = U * E;
+  extern __shared__ __align__(16) uint32_t smem_dyn[];
+  uint32_t* sk = smem_dyn;                      // tile_words keys
+  uint32_t* sv = smem_dyn + tile_words<E, U>(); // tile_words values (pairs only)
+  const int tid = threadIdx.x;
+  const long long t0 = tile * T;
+  const long long rem = args.n - t0;
+  const int cnt = rem < T ? (int)rem : T;
+  tma::pdl_wait();  // the input may be produced by the preceding grid
+  // (after the wait: the preceding grid may be a merge launch using the flags)
+  if (args.zero != nullptr && tile == 0)
+    for (int k = tid; k < args.nzero; k += U) args.zero[k] = 0u;
+  uint32_t key[E], val[E];
+  block_sort_core<E, U, PAIRS, CF>(args, sk, sv, t0, cnt, key, val);
   __syncthreads();
   tma::pdl_trigger();  // the next pass may be scheduled once this wave ends
   // --- store run `tile`: descending iff tile odd (CF directions)
@@ -395,6 +409,134 @@ __device__ __forceinline__ void block_sort_tile(const SortArgs& args, const long
   const long long c0 = desc ? t0 + ((T - cnt) & 3) + cnt - T : t0;
   store_tile<E, U, PAIRS>(sk, sv, key, val, tid * E, cnt, desc, args.out_k, args.out_v, c0,
                           args.decode_f32 != 0);
+}
+
+// ---------------------------------------------------------------------------
+// Two-tile block sort (keys only, CF, E coprime with w; SURVEY.md §8(f) f3,
+// fewer HBM passes): one CTA sorts the tiles 2p and 2p+1 (T = U*E keys each)
+// with block_sort_core, keeps them in shared memory as one merge group of the
+// paper's layout (tile 2p ascending at [0, T), tile 2p+1 reversed (pi) at
+// [T, 2T)), and merges them with one more conflict-free level in two rounds
+// of T outputs (warp origins, lane splits, Alg. 1 gather, register merge):
+// runs of 2T leave the kernel, so the sort needs one merge pass fewer.
+// ---------------------------------------------------------------------------
+template <int E, int U>
+__host__ __device__ constexpr int tile2_words() {
+  return 2 * U * E + E + 1;
+}
+
+template <int E, int U>
+__device__ __forceinline__ void block_sort2_tile(const SortArgs& args, const long long pair) {
+  static_assert(cgcd(W, E) == 1, "two-tile block sort: rho = identity");
+  constexpr int T = U * E;
+  constexpr int T2 = 2 * T;
+  constexpr int NW = U / W;
+  extern __shared__ __align__(16) uint32_t smem_dyn[];
+  uint32_t* sk = smem_dyn;  // tile2_words keys
+  __shared__ int s_org2[2][NW + 1];
+  const int tid = threadIdx.x;
+  const int lane = tid & (W - 1);
+  const int warp = tid >> 5;
+  const long long t0 = pair * T2;
+  const long long rem = args.n - t0;
+  const int cntA = rem < T ? (int)rem : T;
+  const int cntB = rem - T <= 0 ? 0 : (rem - T < T ? (int)(rem - T) : T);
+  tma::pdl_wait();
+  if (args.zero != nullptr && pair == 0)
+    for (int k = tid; k < args.nzero; k += U) args.zero[k] = 0u;
+  uint32_t key[E], val[E];
+  const bool desc = args.cf_dirs && (pair & 1);
+  const int ntile = cntB > 0 ? 2 : 1;
+  // one copy of the block-sort code for both tiles (instruction cache)
+#pragma unroll 1
+  for (int h = 0; h < ntile; ++h) {
+    block_sort_core<E, U, false, true>(args, sk + h * T, sk + h * T, t0 + h * T, h ? cntB : cntA, key, val);
+    __syncthreads();  // every thread has finished reading the tile's buffer
+    if (ntile == 1) break;
+    // tile 2p -> A at [0, T) ascending (round m writes tid E + m, a round
+    // set); tile 2p+1 -> B reversed, B[y] at 2T-1-y (a short B stays anchored
+    // at the group end, reading c17; round m writes 2T-1-tid E-m)
+    const int base = h ? T2 - 1 - tid * E : tid * E;
+    const int step = h ? -1 : 1;
+#pragma unroll
+    for (int m = 0; m < E; ++m) sk[base + step * m] = key[m];
+  }
+  if (ntile == 1) {
+    // the last, short run: one tile
+    tma::pdl_trigger();
+    const long long c0 = desc ? t0 + ((T - cntA) & 3) + cntA - T : t0;
+    store_tile<E, U, false>(sk, sk, key, val, tid * E, cntA, desc, args.out_k, args.out_v, c0,
+                            args.decode_f32 != 0);
+    return;
+  }
+  __syncthreads();
+  // one more CF merge level over the group (NA = T, NB = cntB), two rounds
+  const int NA = T, NB = cntB, cnt2 = T + cntB;
+  uint32_t key0[E];
+#pragma unroll 1
+  for (int r = 0; r < 2; ++r) {
+    const int Dw = r * T + warp * W * E;
+    const int alpha = warp_origin_smem<E>(sk, 0, T2, NA, NB, Dw, lane);
+    if (lane == 0) s_org2[r][warp] = alpha;
+    if (warp == 0) {
+      const int aend = r == 0 ? warp_origin_smem<E>(sk, 0, T2, NA, NB, T, lane) : NA;
+      if (lane == 0) s_org2[r][NW] = aend;
+    }
+    __syncthreads();
+    const int D = r * T + tid * E;
+    int a = lane_split_smem<E>(sk, 0, T2, NA, NB, Dw, alpha, lane, W, 5);
+    if (D >= cnt2) a = NA;
+    int anext = __shfl_down_sync(FULL, a, 1);
+    if (lane == W - 1) anext = (Dw + W * E >= cnt2) ? NA : s_org2[r][warp + 1];
+    const int Dc = D < cnt2 ? D : cnt2;
+    const int Dn = D + E < cnt2 ? D + E : cnt2;
+    const int nA = anext - a;
+    const int nB = (Dn - Dc) - nA;
+    const int b = Dc - a;
+    if (cnt2 == T2)
+      dual_subsequence_gather<E, false, true>(sk, sk, 0, T2, a, b, nA, nB, key, val, PAD_KEY);
+    else
+      dual_subsequence_gather<E, false, false>(sk, sk, 0, T2, a, b, nA, nB, key, val, PAD_KEY);
+    merge_registers<E, false>(key, val, a, nA, nB);
+    if (r == 0) {
+#pragma unroll
+      for (int m = 0; m < E; ++m) key0[m] = key[m];
+    }
+  }
+  __syncthreads();
+  tma::pdl_trigger();
+  // --- store the run of 2T (descending iff the pair index is odd; a short
+  // descending run shifted by sigma = (2T - cnt2) mod 4): round-set STS of
+  // both rounds' outputs, then coalesced stores
+  const int D0 = tid * E, D1 = T + tid * E;
+  if (desc) {
+#pragma unroll
+    for (int m = 0; m < E; ++m) sk[T2 - E - D0 + m] = key0[E - 1 - m];
+#pragma unroll
+    for (int m = 0; m < E; ++m) sk[T2 - E - D1 + m] = key[E - 1 - m];
+  } else {
+#pragma unroll
+    for (int m = 0; m < E; ++m) sk[D0 + m] = key0[m];
+#pragma unroll
+    for (int m = 0; m < E; ++m) sk[D1 + m] = key[m];
+  }
+  __syncthreads();
+  const long long c0 = desc ? t0 + ((T2 - cnt2) & 3) + cnt2 - T2 : t0;
+  const int qlo = desc ? T2 - cnt2 : 0;
+  const int qhi = desc ? T2 : cnt2;
+  uint32_t* __restrict__ pk = args.out_k + c0;
+  if (args.decode_f32) {
+    for (int q = qlo + tid; q < qhi; q += U) pk[q] = f32_decode(sk[q]);
+    return;
+  }
+  // consecutive words per warp: conflict-free loads, coalesced stores
+#pragma unroll 4
+  for (int q = qlo + tid; q < qhi; q += U) pk[q] = sk[q];
+}
+
+template <int E, int U>
+__global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort2_kernel(SortArgs args) {
+  block_sort2_tile<E, U>(args, blockIdx.x);
 }
 
 // ---------------------------------------------------------------------------

@@ -19,6 +19,7 @@ struct Variant {
   MergeFn merge_tma = nullptr;    // persistent TMA pass (CF, E coprime with 32); grid arg = tiles
   MergeFn merge_win = nullptr;    // the persistent window kernel itself (keys or pairs; reads src_kb/src_vb), or nullptr
   MergeFn merge_multi = nullptr;  // the window kernel running MergeArgs::npass regular passes in one launch
+  BlockSortFn block_sort2 = nullptr;  // two-tile block sort (runs of 2 U E; keys-only CF, E = 31)
 };
 
 // [E][u index][algo: 0 CF, 1 baseline][pairs]

@@ -63,6 +63,15 @@ cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s)
   return launch_k(block_sort_kernel<E, U, PAIRS, CF>, (unsigned)grid, U, smem, s, a);
 }
 
+template <int E, int U>
+cudaError_t launch_block_sort2(const SortArgs& a, long long grid, cudaStream_t s) {
+  constexpr size_t smem = (size_t)tile2_words<E, U>() * sizeof(uint32_t);
+  static int done = 0;
+  cudaError_t e = ensure_smem_attr(block_sort2_kernel<E, U>, smem, done);
+  if (e != cudaSuccess) return e;
+  return launch_k(block_sort2_kernel<E, U>, (unsigned)grid, U, smem, s, a);
+}
+
 template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
@@ -177,6 +186,7 @@ void register_eu(LaunchTable& t) {
     if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
       t.v[E][ui][0][1].merge_tma = &launch_merge_win<E, U, true>;
   }
+  if constexpr (cgcd(W, E) == 1 && E + 1 == W && U == 256) t.v[E][ui][0][0].block_sort2 = &launch_block_sort2<E, U>;
   if constexpr (cgcd(W, E) == 1) {
     t.v[E][ui][0][0].merge_tma = &launch_merge_tma<E, U, false>;
     t.v[E][ui][0][1].merge_tma = &launch_merge_tma<E, U, true>;

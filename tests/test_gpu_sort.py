@@ -498,3 +498,26 @@ def test_host_batch_parity(nbatch, n):
     torch.cuda.synchronize()
     for i, x in enumerate(xs):
         np.testing.assert_array_equal(h_in[i].numpy().view(np.uint32), oracle.sort_u32(x), err_msg=f"in place {i}")
+
+
+BS2_SIZES = [1, 7936, 7937, 15871, 15872, 15873, 15872 * 3 + 5, 100003, 1 << 20]
+
+
+@pytest.mark.parametrize("n", BS2_SIZES)
+@pytest.mark.parametrize("kind", ["uniform", "dup", "worst"])
+def test_two_tile_block_sort(n, kind, monkeypatch):
+    """The opt-in two-tile block sort (BCF_BS2=1): runs of 2 x 7936
+    keys (both tiles sorted, then one more CF level in shared memory), one
+    merge pass fewer; the plan reports it and the result is the oracle's."""
+    monkeypatch.setenv("BCF_BS2", "1")
+    plan = bcf.sort_plan(n)
+    assert plan["block_sort_tile"] == 2 * 7936
+    seed = si.config_seed(0) + n
+    if kind == "worst":
+        x = to_host(bcf.worst_case(n, 31, 128, seed=seed, device=DEV))
+    else:
+        x = si.uniform_u32(n, seed) if kind == "uniform" else si.dup_u32(n, seed, mask=0x3)
+    np.testing.assert_array_equal(gpu_sort_u32(x), oracle.sort_u32(x))
+    f = si.special_f32_bits(n, seed)
+    fo = bcf.sort(torch.from_numpy(f.view(np.float32).copy()).to(DEV))
+    np.testing.assert_array_equal(to_host(fo), oracle.sort_f32_bits(f))
