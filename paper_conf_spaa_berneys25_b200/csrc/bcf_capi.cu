@@ -286,6 +286,9 @@ static bcf_status sort_impl(const uint32_t* in_k, uint32_t* out_k, const uint32_
   while ((T << lg_bs) < Tbs) ++lg_bs;
   int P = 0;
   while ((Tbs << P) < (long long)n) ++P;
+#if defined(BCF_TIMING_SKIP_LEVELS) || defined(BCF_TIMING_SKIP_WARP) || defined(BCF_TIMING_BS_ONLY)
+  P = 0;  // timing-only builds: the block sort alone
+#endif
   const bool use_tma = cf && var.merge_tma != nullptr && !tma_disabled();
 
   char* tb = (char*)align_up((size_t)d_temp, 256);

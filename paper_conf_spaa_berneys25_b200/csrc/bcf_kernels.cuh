@@ -283,11 +283,16 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
 #pragma unroll
     for (int i = 0; i < E; ++i) k32[i] = key[i];
     k32[E] = PAD_KEY;
+#ifndef BCF_TIMING_SKIP_WARP
     warp_bitonic_levels(k32, lane);
+#endif
     __syncthreads();  // (general path: every thread has finished its blocked read of sk)
     warp_run_scatter<E>(sk, k32, warp, lane);
     l_first = 5;
   }
+#ifdef BCF_TIMING_SKIP_LEVELS
+  l_first = 30;  // timing-only build: no shared-memory levels (wrong output)
+#endif
 
   // --- log2(U) merge levels: runs of S = E*2^l, groups of G = 2^(l+1) threads
 #pragma unroll 1
