@@ -156,11 +156,26 @@ __device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uin
       if constexpr (PAIRS) sv[idx] = val[m];
     }
   }
-  __syncthreads();
   const int qlo = desc ? T - cnt : 0;
   const int qhi = desc ? T : cnt;
   uint32_t* __restrict__ pk = gk + c0;
   uint32_t* __restrict__ pv = PAIRS ? gv + c0 : nullptr;
+  if constexpr (cgcd(W, E) == 1 && !PAIRS && (T % 4) == 0) {
+    // a full tile of keys to a 16-byte aligned run: one bulk (TMA) store of the
+    // staged tile (rho = identity: physical order is the output order)
+    if (cnt == T && !decode && (((uintptr_t)pk) & 15) == 0) {
+      tma::fence_proxy_async_smem();  // every thread's staging stores, before the async read
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        tma::bulk_s2g(pk, sk, (uint32_t)T * 4u);
+        tma::bulk_commit();
+        tma::bulk_wait_read_all();  // shared memory is read before the CTA moves on / exits
+      }
+      __syncthreads();
+      return;
+    }
+  }
+  __syncthreads();
   if (decode) {
 #pragma unroll
     for (int r = 0; r < E; ++r) {
@@ -225,8 +240,13 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
     const int wbase = warp * (W * E);
     const uint32_t* __restrict__ gin_k = args.in_k + t0 + wbase + lane;
     const int lim = cnt - wbase - lane;  // element 32 r + lane exists iff 32 r < lim
+    if (lim >= W * E) {  // a full warp chunk (every tile but the last): no predicates
 #pragma unroll
-    for (int r = 0; r < E; ++r) key[r] = (W * r < lim) ? __ldg(gin_k + W * r) : PAD_KEY;
+      for (int r = 0; r < E; ++r) key[r] = __ldg(gin_k + W * r);
+    } else {
+#pragma unroll
+      for (int r = 0; r < E; ++r) key[r] = (W * r < lim) ? __ldg(gin_k + W * r) : PAD_KEY;
+    }
     if (args.encode_f32) {
 #pragma unroll
       for (int r = 0; r < E; ++r)
