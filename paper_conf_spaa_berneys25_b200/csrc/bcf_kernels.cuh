@@ -209,9 +209,14 @@ __device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uin
 #ifndef BCF_BS_MINB512
 #define BCF_BS_MINB512 0
 #endif
-template <int U>
+#ifndef BCF_BS_PAIRS_MINB256
+#define BCF_BS_PAIRS_MINB256 5  // pairs (11, 256): <= 51 registers, 5 CTAs/SM (ptxas alone picks 64)
+#endif
+template <int U, bool PAIRS = false, int E = 0>
 __host__ __device__ constexpr int bs_min_blocks() {
-  return U == 256 ? BCF_BS_MINB256 : (U == 512 ? BCF_BS_MINB512 : 0);
+  // (the pairs cap spills at E >= 15: those keep ptxas's choice)
+  return (PAIRS && U == 256 && E <= 13) ? BCF_BS_PAIRS_MINB256
+                                        : (U == 256 ? BCF_BS_MINB256 : (U == 512 ? BCF_BS_MINB512 : 0));
 }
 
 // The block sort of one tile of T = U*E keys (input t0 .. t0+cnt of
@@ -569,7 +574,7 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort2_kernel(Sort
 // runs of R keys.  Group g merges run 2g (A) with run 2g+1 (B).
 // ---------------------------------------------------------------------------
 template <int E, int U, bool PAIRS, bool CF>
-__global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort_kernel(SortArgs args) {
+__global__ void __launch_bounds__(U, bs_min_blocks<U, PAIRS, E>()) block_sort_kernel(SortArgs args) {
   const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
   for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
     if (t != blockIdx.x) __syncthreads();  // the previous tile's copy-out has read shared memory

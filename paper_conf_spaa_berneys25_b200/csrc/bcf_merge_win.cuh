@@ -133,15 +133,21 @@ __device__ __forceinline__ int warp_prefix_count_rho(int n, P pred, int l0, int 
 }
 
 // resident CTAs per SM the kernel is built for (5 at u = 128)
-template <int U, bool PAIRS = false>
+template <int U, bool PAIRS = false, int E = 0>
 __host__ __device__ constexpr int win_min_blocks() {
   // pairs: twice the stage bytes and a value + tag register per key
-  if (PAIRS) return U <= 128 ? 3 : (U <= 256 ? 2 : 1);
+#ifndef BCF_WIN_PAIRS_MINB256
+#define BCF_WIN_PAIRS_MINB256 3  // 3 CTAs/SM at (11, 256): <= 75 registers (the pass loop of the multi-pass mode had raised ptxas's choice to 95, 2 CTAs/SM)
+#endif
+  if (PAIRS) return U <= 128 ? 3 : (U <= 256 ? (E <= 13 ? BCF_WIN_PAIRS_MINB256 : 2) : 1);
   return WIN_STAGES > 2 ? (U <= 128 ? 3 : 1) : (U <= 128 ? 5 : (U <= 256 ? 2 : 1));
 }
 
-template <int E, int U, bool PAIRS = false>
-__global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass_win_kernel(MergeArgs args, long long tiles,
+// MULTI: the multi-pass instantiation (MergeArgs::npass passes in one launch);
+// the one-pass kernel does not carry its machinery (registers: (11, 256)
+// pairs 95 -> 72, (11, 256) keys 88 -> 64)
+template <int E, int U, bool PAIRS = false, bool MULTI = false>
+__global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS, E>()) merge_pass_win_kernel(MergeArgs args, long long tiles,
                                                                 long long per_cta) {
   constexpr int T = U * E;
   constexpr int S2 = win_span<E, U>();
@@ -169,8 +175,8 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS>()) merge_pass
   if (t_end <= t_begin) return;
   // multi-pass mode: passes p = 0..npass-1 of a sort in this one launch
   // (MergeArgs::npass); a CTA keeps its tile range in every pass
-  const bool multi = args.npass > 1;
-  const int npass = multi ? args.npass : 1;
+  constexpr bool multi = MULTI;
+  const int npass = MULTI ? args.npass : 1;
   auto pass_args = [&](int p) {
     MergeArgs a = args;
     if (multi) {

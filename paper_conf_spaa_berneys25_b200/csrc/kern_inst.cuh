@@ -165,7 +165,7 @@ cudaError_t launch_merge_win(const MergeArgs& a, long long tiles, cudaStream_t s
 template <int E, int U, bool PAIRS>
 cudaError_t launch_merge_multi(const MergeArgs& a, long long tiles, cudaStream_t s) {
   static PersistentCache pc;
-  return launch_persistent(merge_pass_win_kernel<E, U, PAIRS>, pc, win_smem_bytes<E, U, PAIRS>(), U + 32, a, tiles,
+  return launch_persistent(merge_pass_win_kernel<E, U, PAIRS, true>, pc, win_smem_bytes<E, U, PAIRS>(), U + 32, a, tiles,
                            s);
 }
 
