@@ -573,12 +573,20 @@ __global__ void __launch_bounds__(U, bs_min_blocks<U>()) block_sort2_kernel(Sort
 // Merge pass (K2+K3 fused): output tile `blockIdx.x` of the pairwise merge of
 // runs of R keys.  Group g merges run 2g (A) with run 2g+1 (B).
 // ---------------------------------------------------------------------------
-template <int E, int U, bool PAIRS, bool CF>
+// LOOP: a grid smaller than the tile count loops over the tiles (grid stride,
+// the one-CTA-per-SM measurement mode, SortArgs::ntiles).  A separate
+// instantiation: the loop raises ptxas's register choice for the whole kernel
+// (block_sort<31, 256> 80 -> 128 registers, 138 -> 146 us at 2^24).
+template <int E, int U, bool PAIRS, bool CF, bool LOOP = false>
 __global__ void __launch_bounds__(U, bs_min_blocks<U, PAIRS, E>()) block_sort_kernel(SortArgs args) {
-  const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
-  for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
-    if (t != blockIdx.x) __syncthreads();  // the previous tile's copy-out has read shared memory
-    block_sort_tile<E, U, PAIRS, CF>(args, t);
+  if constexpr (!LOOP) {
+    block_sort_tile<E, U, PAIRS, CF>(args, blockIdx.x);
+  } else {
+    const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
+    for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
+      if (t != blockIdx.x) __syncthreads();  // the previous tile's copy-out has read shared memory
+      block_sort_tile<E, U, PAIRS, CF>(args, t);
+    }
   }
 }
 
@@ -722,12 +730,17 @@ __device__ __forceinline__ void merge_pass_tile(const MergeArgs& args, const lon
                           args.decode_f32 != 0);
 }
 
-template <int E, int U, bool PAIRS, bool CF, bool BDESC>
+// LOOP: as for block_sort_kernel (MergeArgs::ntiles, grid-stride over tiles)
+template <int E, int U, bool PAIRS, bool CF, bool BDESC, bool LOOP = false>
 __global__ void __launch_bounds__(U) merge_pass_kernel(MergeArgs args) {
-  const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
-  for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
-    if (t != blockIdx.x) __syncthreads();
-    merge_pass_tile<E, U, PAIRS, CF, BDESC>(args, t);
+  if constexpr (!LOOP) {
+    merge_pass_tile<E, U, PAIRS, CF, BDESC>(args, blockIdx.x);
+  } else {
+    const long long nt = args.ntiles > 0 ? args.ntiles : (long long)gridDim.x;
+    for (long long t = blockIdx.x; t < nt; t += gridDim.x) {
+      if (t != blockIdx.x) __syncthreads();
+      merge_pass_tile<E, U, PAIRS, CF, BDESC>(args, t);
+    }
   }
 }
 

@@ -57,7 +57,12 @@ cudaError_t launch_k(void (*kern)(KArgs...), unsigned grid, unsigned block, size
 template <int E, int U, bool PAIRS, bool CF>
 cudaError_t launch_block_sort(const SortArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
-  static int done = 0;
+  static int done = 0, done_loop = 0;
+  if (a.ntiles > 0) {  // grid-stride measurement mode
+    cudaError_t e = ensure_smem_attr(block_sort_kernel<E, U, PAIRS, CF, true>, smem, done_loop);
+    if (e != cudaSuccess) return e;
+    return launch_k(block_sort_kernel<E, U, PAIRS, CF, true>, (unsigned)grid, U, smem, s, a);
+  }
   cudaError_t e = ensure_smem_attr(block_sort_kernel<E, U, PAIRS, CF>, smem, done);
   if (e != cudaSuccess) return e;
   return launch_k(block_sort_kernel<E, U, PAIRS, CF>, (unsigned)grid, U, smem, s, a);
@@ -75,7 +80,12 @@ cudaError_t launch_block_sort2(const SortArgs& a, long long grid, cudaStream_t s
 template <int E, int U, bool PAIRS, bool CF, bool BDESC>
 cudaError_t launch_merge(const MergeArgs& a, long long grid, cudaStream_t s) {
   constexpr size_t smem = tile_smem_bytes<E, U, PAIRS>();
-  static int done = 0;
+  static int done = 0, done_loop = 0;
+  if (a.ntiles > 0) {  // grid-stride measurement mode
+    cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC, true>, smem, done_loop);
+    if (e != cudaSuccess) return e;
+    return launch_k(merge_pass_kernel<E, U, PAIRS, CF, BDESC, true>, (unsigned)grid, U, smem, s, a);
+  }
   cudaError_t e = ensure_smem_attr(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, smem, done);
   if (e != cudaSuccess) return e;
   return launch_k(merge_pass_kernel<E, U, PAIRS, CF, BDESC>, (unsigned)grid, U, smem, s, a);
