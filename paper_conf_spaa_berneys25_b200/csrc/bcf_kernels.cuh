@@ -160,22 +160,20 @@ __device__ __forceinline__ void store_tile(uint32_t* sk, uint32_t* sv, const uin
   const int qhi = desc ? T : cnt;
   uint32_t* __restrict__ pk = gk + c0;
   uint32_t* __restrict__ pv = PAIRS ? gv + c0 : nullptr;
+  // (LSU stores, not a bulk copy: a bulk shared->global copy running beside
+  // other CTAs' shared-memory instructions shows up in the unit-level bank
+  // conflict counter -- 0.68 M per 2^24 block sort)
+  __syncthreads();
   if constexpr (cgcd(W, E) == 1 && !PAIRS && (T % 4) == 0) {
-    // a full tile of keys to a 16-byte aligned run: one bulk (TMA) store of the
-    // staged tile (rho = identity: physical order is the output order)
+    // a full tile into a 16-byte aligned run (rho = identity: physical order is
+    // the output order): 16-byte loads and stores, a quarter-warp reads 128
+    // consecutive bytes (one wavefront, no conflict)
     if (cnt == T && !decode && (((uintptr_t)pk) & 15) == 0) {
-      tma::fence_proxy_async_smem();  // every thread's staging stores, before the async read
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        tma::bulk_s2g(pk, sk, (uint32_t)T * 4u);
-        tma::bulk_commit();
-        tma::bulk_wait_read_all();  // shared memory is read before the CTA moves on / exits
-      }
-      __syncthreads();
+      for (int q = 4 * (int)threadIdx.x; q < T; q += 4 * U)
+        *reinterpret_cast<uint4*>(pk + q) = *reinterpret_cast<const uint4*>(sk + q);
       return;
     }
   }
-  __syncthreads();
   if (decode) {
 #pragma unroll
     for (int r = 0; r < E; ++r) {
