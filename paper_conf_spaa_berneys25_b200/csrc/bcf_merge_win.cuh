@@ -175,8 +175,9 @@ __global__ void __launch_bounds__(U + 32, win_min_blocks<U, PAIRS, E>()) merge_p
   if (t_end <= t_begin) return;
   // multi-pass mode: passes p = 0..npass-1 of a sort in this one launch
   // (MergeArgs::npass); a CTA keeps its tile range in every pass
-  constexpr bool multi = MULTI;
-  const int npass = MULTI ? args.npass : 1;
+  // (MULTI instantiation: the multi-pass machinery, used when args.npass > 1)
+  const bool multi = MULTI && args.npass > 1;
+  const int npass = multi ? args.npass : 1;
   auto pass_args = [&](int p) {
     MergeArgs a = args;
     if (multi) {

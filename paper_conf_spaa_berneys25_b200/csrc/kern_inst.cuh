@@ -179,6 +179,11 @@ cudaError_t launch_merge_multi(const MergeArgs& a, long long tiles, cudaStream_t
                            s);
 }
 
+inline bool even_window_enabled() {
+  const char* v = getenv("BCF_EVEN_WIN");
+  return v && v[0] == '1';
+}
+
 template <int E, int U>
 void register_eu(LaunchTable& t) {
   const int ui = u_index(U);
@@ -190,11 +195,17 @@ void register_eu(LaunchTable& t) {
                       nullptr};
   if constexpr (cgcd(W, E) > 1) {
     // rho != identity: the window kernel with cp.async staging in rho's
-    // physical order and LSU copy-out (regular passes and merge_runs passes)
-    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
-      t.v[E][ui][0][0].merge_tma = &launch_merge_win<E, U, false>;
-    if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
-      t.v[E][ui][0][1].merge_tma = &launch_merge_win<E, U, true>;
+    // physical order and LSU copy-out is opt-in (BCF_EVEN_WIN=1): the one-CTA-
+    // per-tile kernel with physical-order LSU staging by every thread is faster
+    // for every even E (2^27: 530-800 vs 800-2240 us per pass,
+    // profiles/r02_evenE_plain_vs_window_2p27.txt).  (The general (MULTI)
+    // instantiation: faster here than the one-pass one, 795 vs 875 us.)
+    if (even_window_enabled()) {
+      if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U>() <= 227 * 1024)
+        t.v[E][ui][0][0].merge_tma = &launch_merge_multi<E, U, false>;
+      if constexpr (BCF_MERGE_WIN && win_smem_bytes<E, U, true>() <= 227 * 1024)
+        t.v[E][ui][0][1].merge_tma = &launch_merge_multi<E, U, true>;
+    }
   }
   if constexpr (cgcd(W, E) == 1 && E + 1 == W && U == 256) t.v[E][ui][0][0].block_sort2 = &launch_block_sort2<E, U>;
   if constexpr (cgcd(W, E) == 1) {

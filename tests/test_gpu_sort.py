@@ -521,3 +521,38 @@ def test_two_tile_block_sort(n, kind, monkeypatch):
     f = si.special_f32_bits(n, seed)
     fo = bcf.sort(torch.from_numpy(f.view(np.float32).copy()).to(DEV))
     np.testing.assert_array_equal(to_host(fo), oracle.sort_f32_bits(f))
+
+
+def test_even_e_window_kernel_opt_in():
+    """The persistent window kernel for even E (cp.async staging in rho's
+    physical order; opt-in BCF_EVEN_WIN=1, read when the launch table is
+    built): a fresh process sorts keys and stable pairs at every even E
+    against the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = r'''
+import sys
+sys.path.insert(0, %r)
+import numpy as np, torch
+import oracle, synthetic_inputs as si, paper_conf_spaa_berneys25_b200 as bcf
+dev = torch.device("cuda:0")
+n = 90001
+x = si.dup_u32(n, 11, mask=0xFFF)
+v = si.iota_u32(n)
+for E in (8, 10, 12, 14, 16):
+    for u in (128, 256):
+        p = bcf.make_params(E, u)
+        out = bcf.sort(torch.from_numpy(x.view(np.int32).copy()).to(dev), params=p)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), oracle.sort_u32(x)), (E, u)
+        ko, vo = bcf.sort_pairs(torch.from_numpy(x.view(np.int32).copy()).to(dev),
+                                torch.from_numpy(v.view(np.int32).copy()).to(dev), params=p)
+        ek, ev = oracle.sort_pairs_u32(x, v)
+        assert np.array_equal(ko.cpu().numpy().view(np.uint32), ek), (E, u, "pairs keys")
+        assert np.array_equal(vo.cpu().numpy().view(np.uint32), ev), (E, u, "pairs values")
+print("even-window ok")
+''' % root
+    env = dict(os.environ, BCF_EVEN_WIN="1")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "even-window ok" in r.stdout, r.stdout + r.stderr
