@@ -656,15 +656,16 @@ __device__ __forceinline__ uint32_t lane_minmax(uint32_t a, uint32_t p, bool hi,
   return hi ? max(a, p) : min(a, p);
 }
 
-__device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[W], int lane) {
+template <int NS = W>
+__device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[NS], int lane) {
 #pragma unroll
   for (int L = 0; L < 5; ++L) {
     const bool up = (lane >> L) & 1;
     const uint32_t up01 = up ? 1u : 0u;
     const int m = (2 << L) - 1;
 #pragma unroll
-    for (int i = 0; i < W / 2; ++i) {
-      const int j = W - 1 - i;
+    for (int i = 0; i < NS / 2; ++i) {
+      const int j = NS - 1 - i;
       const uint32_t pi = __shfl_xor_sync(FULL, k[j], m);
       const uint32_t pj = __shfl_xor_sync(FULL, k[i], m);
       k[i] = lane_minmax(k[i], pi, up, up01, false);
@@ -675,13 +676,13 @@ __device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[W], int lane) 
       const bool hi = (lane >> d) & 1;
       const uint32_t hi01 = hi ? 1u : 0u;
 #pragma unroll
-      for (int i = 0; i < W; ++i) {
+      for (int i = 0; i < NS; ++i) {
         const uint32_t p = __shfl_xor_sync(FULL, k[i], 1 << d);
         k[i] = lane_minmax(k[i], p, hi, hi01, (i & 1) != 0);
       }
     }
-    uint32_t dt[W], dv[W];
-    bitonic_merge_pad<W, false>(k, dt, dv);
+    uint32_t dt[NS], dv[NS];
+    bitonic_merge_pad<NS, false>(k, dt, dv);
   }
 }
 
@@ -723,6 +724,22 @@ __device__ __forceinline__ void warp_run_scatter(uint32_t* __restrict__ sk, cons
       *reinterpret_cast<uint4*>(sk + gbase + W * lane + 4 * qq) = v;
     }
   }
+}
+
+// The same write for E = 16 or 8 (E slots per lane, no pads, rho != identity):
+// lane i of warp run holds run positions [E i, E i + E); round r writes
+// position E i + r (A, ascending) or its mirror 2S-1-(E i + r) (B, pi), a
+// round set of the run's wE window (Lemma 1 / Cor. 3): conflict-free via rho.
+template <int E>
+__device__ __forceinline__ void warp_run_scatter_rho(uint32_t* __restrict__ sk, const uint32_t (&k)[E], int warp,
+                                                     int lane) {
+  constexpr int S = W * E;
+  const int gbase = (warp >> 1) * 2 * S;
+  const bool isB = warp & 1;
+  const int base = isB ? gbase + 2 * S - 1 - E * lane : gbase + E * lane;
+  const int step = isB ? -1 : 1;
+#pragma unroll
+  for (int r = 0; r < E; ++r) sk[rho<E>(base + step * r)] = k[r];
 }
 
 // f32 <-> order-preserving u32 (IEEE totalOrder, reading c2)

@@ -222,6 +222,9 @@ __host__ __device__ constexpr int bs_min_blocks() {
 // outputs [tid E, tid E + E) in key[] (val[] for pairs); sk / sv (tile_words
 // each) are its working buffers, still being read by other threads until the
 // caller's next __syncthreads.
+#ifndef BCF_WARP_POW2
+#define BCF_WARP_POW2 1
+#endif
 template <int E, int U, bool PAIRS, bool CF>
 __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* sk, uint32_t* sv,
                                                 const long long t0, const int cnt, uint32_t (&key)[E],
@@ -237,7 +240,9 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
   // keys to its lanes works, so each lane loads its keys straight from global
   // memory (coalesced: key r of lane l is element 32 r + l of the warp's
   // chunk) without the shared-memory round trip of the general path
-  constexpr bool WARP_PHASE = CF && !PAIRS && E + 1 == W && U >= 2 * W;
+  // (also E = 16 and 8: E slots per lane, no pad, the warp runs written
+  // through rho; BCF_WARP_POW2=0 keeps those on the shared-memory levels)
+  constexpr bool WARP_PHASE = CF && !PAIRS && U >= 2 * W && (E + 1 == W || (BCF_WARP_POW2 && (E == 16 || E == 8)));
   uint32_t tag[E];
   if constexpr (WARP_PHASE) {
     const int wbase = warp * (W * E);
@@ -301,16 +306,21 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
   // warp phase, then the warp runs go to shared memory in the level-5 layout
   // and the CF shared-memory levels continue from l = 5
   int l_first = 0;
-  if constexpr (WARP_PHASE) {
+  if constexpr (WARP_PHASE && E + 1 == W) {
     uint32_t k32[W];
 #pragma unroll
     for (int i = 0; i < E; ++i) k32[i] = key[i];
     k32[E] = PAD_KEY;
 #ifndef BCF_TIMING_SKIP_WARP
-    warp_bitonic_levels(k32, lane);
+    warp_bitonic_levels<W>(k32, lane);
 #endif
     __syncthreads();  // (general path: every thread has finished its blocked read of sk)
     warp_run_scatter<E>(sk, k32, warp, lane);
+    l_first = 5;
+  } else if constexpr (WARP_PHASE) {
+    warp_bitonic_levels<E>(key, lane);
+    __syncthreads();
+    warp_run_scatter_rho<E>(sk, key, warp, lane);
     l_first = 5;
   }
 #ifdef BCF_TIMING_SKIP_LEVELS
