@@ -395,6 +395,20 @@ __device__ __forceinline__ uint32_t imad_u32(uint32_t a, uint32_t b, uint32_t c)
   return r;
 }
 
+// which compare-exchanges take the FMA form (A/B builds: BCF_FMA_MOD = m puts
+// the max of (m-1) of every m exchanges on the FMA pipe, 0 = none;
+// BCF_LANE_FMA_MOD likewise for the cross-lane half-cleaner selects)
+#ifndef BCF_FMA_MOD
+#define BCF_FMA_MOD 3
+#endif
+#ifndef BCF_LANE_FMA_MOD
+#define BCF_LANE_FMA_MOD 2
+#endif
+__host__ __device__ constexpr bool fma_pick(int i) { return BCF_FMA_MOD > 0 && (i % (BCF_FMA_MOD > 0 ? BCF_FMA_MOD : 1)) != 0; }
+__host__ __device__ constexpr bool lane_fma_pick(int i) {
+  return BCF_LANE_FMA_MOD > 0 && (i % (BCF_LANE_FMA_MOD > 0 ? BCF_LANE_FMA_MOD : 1)) != 0;
+}
+
 __device__ __forceinline__ void ce_keys(uint32_t& x, uint32_t& y, bool fma_max) {
   const uint32_t a = x, b = y;
   const uint32_t m = min(a, b);
@@ -460,7 +474,7 @@ __device__ __forceinline__ void bitonic_merge_pad(uint32_t (&k)[E], uint32_t (&t
         const bool vi = (virt >> i) & 1u, vj = (virt >> j) & 1u;
         if (!vi && !vj) {
           if constexpr (PAIRS) Elem<PAIRS>::ce(K[i], K[j], Tg[i], Tg[j], V[i], V[j]);
-          else ce_keys(K[i], K[j], (i % 3) != 0);  // compile-time after unrolling
+          else ce_keys(K[i], K[j], fma_pick(i));  // compile-time after unrolling
         } else if (!vi && vj) {
           // min(-inf, x) = -inf goes to i, x moves to j
           K[j] = K[i];
@@ -509,7 +523,7 @@ __device__ __forceinline__ void oddeven_sort_pad(uint32_t (&k)[E], uint32_t (&t)
           const bool vx = (virt >> x) & 1u, vy = (virt >> y) & 1u;
           if (!vx && !vy) {
             if constexpr (PAIRS) Elem<PAIRS>::ce(K[x], K[y], Tg[x], Tg[y], V[x], V[y]);
-            else ce_keys(K[x], K[y], (x % 3) != 0);
+            else ce_keys(K[x], K[y], fma_pick(x));
           } else if (vx && !vy) {
             // max(+inf, y) = +inf goes to y, y's value moves to x
             K[x] = K[y];
@@ -678,7 +692,7 @@ __device__ __forceinline__ void warp_bitonic_levels(uint32_t (&k)[NS], int lane)
 #pragma unroll
       for (int i = 0; i < NS; ++i) {
         const uint32_t p = __shfl_xor_sync(FULL, k[i], 1 << d);
-        k[i] = lane_minmax(k[i], p, hi, hi01, (i & 1) != 0);
+        k[i] = lane_minmax(k[i], p, hi, hi01, lane_fma_pick(i));
       }
     }
     uint32_t dt[NS], dv[NS];
