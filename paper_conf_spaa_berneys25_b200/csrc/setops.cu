@@ -24,6 +24,9 @@
 namespace bcf {
 namespace setops {
 
+#ifndef BCF_LB_SLEEP_NS
+#define BCF_LB_SLEEP_NS 100
+#endif
 constexpr int THREADS = 256;
 constexpr int ITEMS = 16;
 constexpr long long BLK = (long long)THREADS * ITEMS;
@@ -83,45 +86,62 @@ __device__ __forceinline__ long long first_b(const uint32_t* __restrict__ V, lon
   return lo;
 }
 
-__device__ __forceinline__ bool keep(int op, const uint32_t* __restrict__ M, const uint32_t* __restrict__ V,
-                                     long long n, long long p) {
-  const uint32_t x = __ldg(M + p);
-  const bool isB = (__ldg(V + p) & 0x80000000u) != 0;
-  // fast path: a run of one (no equal neighbour)
-  const bool left = p > 0 && __ldg(M + p - 1) == x;
-  const bool right = p + 1 < n && __ldg(M + p + 1) == x;
-  long long p0, p1, pb;
-  if (!left && !right) {
-    p0 = p;
-    p1 = p + 1;
-    pb = isB ? p : p + 1;
-  } else {
-    p0 = left ? run_begin(M, p, x) : p;
-    p1 = right ? run_end(M, n, p, x) : p + 1;
-    pb = first_b(V, p0, p1);
-  }
-  const long long m = pb - p0, nB = p1 - pb;  // copies in A, in B
+
+// the keep rule for a copy at merged position p of the run [p0, p1) whose B
+// copies start at pb (m = pb - p0 copies from A, nB = p1 - pb from B)
+__device__ __forceinline__ bool keep_rule(int op, bool isB, long long p, long long p0, long long pb, long long p1) {
+  const long long m = pb - p0, nB = p1 - pb;
   if (!isB) {
     const long long k = p - p0;
-    switch (op) {
-      case 0: return true;
-      case 1: return k < nB;
-      default: return k >= nB;  // difference, symmetric difference
-    }
+    return op == 0 ? true : (op == 1 ? k < nB : k >= nB);
   }
-  const long long k = p - pb;
-  return (op == 0 || op == 3) && k >= m;
+  return (op == 0 || op == 3) && p - pb >= m;
 }
 
 // keep bits of a block's BLK merged positions, striped: bit q of thread t is
-// position base + q * THREADS + t (every load of a row is coalesced)
+// position base + q * THREADS + t (every load of a row is coalesced).  A warp
+// row covers 32 consecutive positions: the run bounds and the A/B boundary of
+// a run that starts and ends inside the row come from three ballots (run
+// heads, run tails, B copies); only runs crossing the row's edge search
+// global memory (run_begin / run_end / first_b).
 __device__ __forceinline__ uint32_t keep_bits(int op, const uint32_t* __restrict__ M, const uint32_t* __restrict__ V,
                                               long long n, long long base) {
+  const unsigned lane = threadIdx.x & 31;
   uint32_t mask = 0;
 #pragma unroll 4
   for (int q = 0; q < ITEMS; ++q) {
     const long long p = base + (long long)q * THREADS + threadIdx.x;
-    if (p < n && keep(op, M, V, n, p)) mask |= 1u << q;
+    const long long row0 = p - lane;  // position of the row's lane 0
+    const bool in = p < n;
+    const uint32_t x = in ? __ldg(M + p) : 0u;
+    const bool isB = in && (__ldg(V + p) & 0x80000000u) != 0;
+    uint32_t xp = __shfl_up_sync(0xffffffffu, x, 1);
+    uint32_t xn = __shfl_down_sync(0xffffffffu, x, 1);
+    if (lane == 0) xp = (in && p > 0) ? __ldg(M + p - 1) : ~x;
+    if (lane == 31 || p + 1 >= n) xn = (in && p + 1 < n) ? __ldg(M + p + 1) : ~x;
+    const bool head = in && (p == 0 || xp != x);
+    const bool tail = in && (p + 1 == n || xn != x);
+    const unsigned H = __ballot_sync(0xffffffffu, head);
+    const unsigned Tl = __ballot_sync(0xffffffffu, tail);
+    const unsigned Bm = __ballot_sync(0xffffffffu, isB);
+    if (!in) continue;
+    const unsigned upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);  // lanes 0..lane
+    const unsigned hs = H & upto, te = Tl & ~((1u << lane) - 1u);
+    long long p0, p1, pb;
+    if (hs && te) {
+      const int l0 = 31 - __clz(hs), l1 = __ffs(te) - 1;  // run = lanes [l0, l1]
+      p0 = row0 + l0;
+      p1 = row0 + l1 + 1;
+      const unsigned inrun = (l1 == 31 ? 0xffffffffu : ((2u << l1) - 1u)) & ~((1u << l0) - 1u);
+      const unsigned b = Bm & inrun;
+      pb = b ? row0 + (__ffs(b) - 1) : p1;
+    } else {
+      // the run crosses the row's edge: bounds from global memory
+      p0 = hs ? row0 + (31 - __clz(hs)) : run_begin(M, p, x);
+      p1 = te ? row0 + __ffs(te) : run_end(M, n, p, x);
+      pb = first_b(V, p0, p1);
+    }
+    if (keep_rule(op, isB, p, p0, pb, p1)) mask |= 1u << q;
   }
   return mask;
 }
@@ -202,7 +222,10 @@ __global__ void __launch_bounds__(THREADS) compact_lookback_kernel(int op, const
         const unsigned pre = __ballot_sync(0xffffffffu, (w & ~ST_VAL) == ST_PRE);
         const int first_pre = pre ? __ffs(pre) - 1 : 32;  // nearest prefix in the window
         const unsigned need = first_pre < 31 ? ((2u << first_pre) - 1u) : 0xffffffffu;
-        if ((ready & need) != need) continue;  // a predecessor not yet published: re-read
+        if ((ready & need) != need) {  // a predecessor not yet published: back off, re-read
+          __nanosleep(BCF_LB_SLEEP_NS);
+          continue;
+        }
         unsigned long long add = (lane <= first_pre && k >= 0) ? (w & ST_VAL) : 0ull;
         for (int o = 16; o > 0; o >>= 1) add += __shfl_xor_sync(0xffffffffu, add, o);
         excl += add;
