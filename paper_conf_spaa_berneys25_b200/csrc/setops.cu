@@ -28,7 +28,10 @@ namespace setops {
 #define BCF_LB_SLEEP_NS 100
 #endif
 constexpr int THREADS = 256;
-constexpr int ITEMS = 16;
+#ifndef BCF_SETOP_ITEMS
+#define BCF_SETOP_ITEMS 16
+#endif
+constexpr int ITEMS = BCF_SETOP_ITEMS;
 constexpr long long BLK = (long long)THREADS * ITEMS;
 
 __global__ void tags_kernel(uint32_t* __restrict__ ta, long long na, uint32_t* __restrict__ tb, long long nb) {
