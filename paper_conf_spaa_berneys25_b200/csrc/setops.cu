@@ -27,7 +27,10 @@ namespace setops {
 #ifndef BCF_LB_SLEEP_NS
 #define BCF_LB_SLEEP_NS 100
 #endif
-constexpr int THREADS = 256;
+#ifndef BCF_SETOP_THREADS
+#define BCF_SETOP_THREADS 256
+#endif
+constexpr int THREADS = BCF_SETOP_THREADS;
 #ifndef BCF_SETOP_ITEMS
 #define BCF_SETOP_ITEMS 16
 #endif
@@ -109,42 +112,53 @@ __device__ __forceinline__ bool keep_rule(int op, bool isB, long long p, long lo
 // global memory (run_begin / run_end / first_b).
 __device__ __forceinline__ uint32_t keep_bits(int op, const uint32_t* __restrict__ M, const uint32_t* __restrict__ V,
                                               long long n, long long base) {
-  const unsigned lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31;
+  const bool full = base + BLK <= n;      // every position of the block exists (all but the last block)
+  const bool after_ok = base + BLK < n;   // the position after the block exists
+  const uint32_t* __restrict__ Mb = M + base;
+  const uint32_t* __restrict__ Vb = V + base;
   uint32_t mask = 0;
 #pragma unroll 4
   for (int q = 0; q < ITEMS; ++q) {
-    const long long p = base + (long long)q * THREADS + threadIdx.x;
-    const long long row0 = p - lane;  // position of the row's lane 0
-    const bool in = p < n;
-    const uint32_t x = in ? __ldg(M + p) : 0u;
-    const bool isB = in && (__ldg(V + p) & 0x80000000u) != 0;
+    const int o = q * THREADS + (int)threadIdx.x;  // offset in the block
+    const bool in = full || base + o < n;
+    const uint32_t x = in ? __ldg(Mb + o) : 0u;
+    const bool isB = in && (__ldg(Vb + o) & 0x80000000u) != 0;
     uint32_t xp = __shfl_up_sync(0xffffffffu, x, 1);
     uint32_t xn = __shfl_down_sync(0xffffffffu, x, 1);
-    if (lane == 0) xp = (in && p > 0) ? __ldg(M + p - 1) : ~x;
-    if (lane == 31 || p + 1 >= n) xn = (in && p + 1 < n) ? __ldg(M + p + 1) : ~x;
-    const bool head = in && (p == 0 || xp != x);
-    const bool tail = in && (p + 1 == n || xn != x);
+    if (lane == 0) xp = (in && (o > 0 || base > 0)) ? __ldg(Mb + o - 1) : ~x;
+    const bool next_ok = full ? (o + 1 < BLK || after_ok) : (base + o + 1 < n);
+    if (lane == 31 || !next_ok) xn = (in && next_ok) ? __ldg(Mb + o + 1) : ~x;
+    const bool head = in && xp != x;  // (xp = ~x before position 0)
+    const bool tail = in && xn != x;  // (xn = ~x after position n-1)
     const unsigned H = __ballot_sync(0xffffffffu, head);
     const unsigned Tl = __ballot_sync(0xffffffffu, tail);
     const unsigned Bm = __ballot_sync(0xffffffffu, isB);
     if (!in) continue;
     const unsigned upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);  // lanes 0..lane
     const unsigned hs = H & upto, te = Tl & ~((1u << lane) - 1u);
-    long long p0, p1, pb;
+    bool k;
     if (hs && te) {
-      const int l0 = 31 - __clz(hs), l1 = __ffs(te) - 1;  // run = lanes [l0, l1]
-      p0 = row0 + l0;
-      p1 = row0 + l1 + 1;
+      // the run is lanes [l0, l1] of this row; its B copies start at lane lb
+      const int l0 = 31 - __clz(hs), l1 = __ffs(te) - 1;
       const unsigned inrun = (l1 == 31 ? 0xffffffffu : ((2u << l1) - 1u)) & ~((1u << l0) - 1u);
-      const unsigned b = Bm & inrun;
-      pb = b ? row0 + (__ffs(b) - 1) : p1;
+      const unsigned bb = Bm & inrun;
+      const int lb = bb ? __ffs(bb) - 1 : l1 + 1;
+      if (isB) {
+        k = (op == 0 || op == 3) && lane - lb >= lb - l0;
+      } else {
+        const int kk = lane - l0, nB = l1 + 1 - lb;
+        k = op == 0 ? true : (op == 1 ? kk < nB : kk >= nB);
+      }
     } else {
       // the run crosses the row's edge: bounds from global memory
-      p0 = hs ? row0 + (31 - __clz(hs)) : run_begin(M, p, x);
-      p1 = te ? row0 + __ffs(te) : run_end(M, n, p, x);
-      pb = first_b(V, p0, p1);
+      const long long p = base + o, row0 = p - lane;
+      const long long p0 = hs ? row0 + (31 - __clz(hs)) : run_begin(M, p, x);
+      const long long p1 = te ? row0 + __ffs(te) : run_end(M, n, p, x);
+      const long long pb = first_b(V, p0, p1);
+      k = keep_rule(op, isB, p, p0, pb, p1);
     }
-    if (keep_rule(op, isB, p, p0, pb, p1)) mask |= 1u << q;
+    if (k) mask |= 1u << q;
   }
   return mask;
 }
@@ -165,7 +179,10 @@ __device__ __forceinline__ void st_rel(unsigned long long* p, unsigned long long
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-__global__ void __launch_bounds__(THREADS) compact_lookback_kernel(int op, const uint32_t* __restrict__ M,
+#ifndef BCF_SETOP_MINB
+#define BCF_SETOP_MINB 8  // 8 blocks per SM (32 registers): the look-back waits are latency, more blocks hide them (858 -> 745 us at 2 x 2^25)
+#endif
+__global__ void __launch_bounds__(THREADS, BCF_SETOP_MINB) compact_lookback_kernel(int op, const uint32_t* __restrict__ M,
                                                                    const uint32_t* __restrict__ V, long long n,
                                                                    unsigned long long* __restrict__ status,
                                                                    unsigned int* __restrict__ ticket,
