@@ -196,8 +196,8 @@ bcf_status bcf_ipc_close(void* d_base);
    graph, like the sorts -- after one earlier uncaptured call with the same
    (E, u) on the device: the first launch of each kernel sets its shared
    memory attribute and queries its occupancy, which capture does not allow.
-   bcf_merge_runs_u32 stages its descriptor table with a pageable H2D copy
-   and cannot be captured. */
+   bcf_merge_runs_u32 writes its per-pass descriptor tables with small
+   kernels too and is capturable under the same condition. */
 bcf_status bcf_merge_u32(const uint32_t* d_a, uint64_t na, const uint32_t* d_b, uint64_t nb,
                          const uint32_t* d_a_vals, const uint32_t* d_b_vals, uint32_t* d_out,
                          uint32_t* d_out_vals, void* d_temp, size_t* temp_bytes, const bcf_params* p,

@@ -575,6 +575,28 @@ bcf_status bcf_split_counts_u32(const uint32_t* d_sorted, uint64_t n, const uint
 // into a CUDA graph)
 __global__ void write_desc_kernel(GroupDesc* d, GroupDesc g) { *d = g; }
 
+// bcf_merge_runs_u32's per-pass descriptor tables, likewise written from
+// kernel parameters (chunks of DESC_CHUNK descriptors, one thread each)
+constexpr int DESC_CHUNK = 24;
+struct DescChunk {
+  GroupDesc g[DESC_CHUNK];
+  int count;
+};
+__global__ void write_table_kernel(GroupDesc* d, DescChunk c) {
+  if ((int)threadIdx.x < c.count) d[threadIdx.x] = c.g[threadIdx.x];
+}
+static cudaError_t write_table(GroupDesc* d, const std::vector<GroupDesc>& tab, cudaStream_t s) {
+  for (size_t i = 0; i < tab.size(); i += DESC_CHUNK) {
+    DescChunk c;
+    c.count = (int)std::min<size_t>(DESC_CHUNK, tab.size() - i);
+    for (int j = 0; j < c.count; ++j) c.g[j] = tab[i + j];
+    write_table_kernel<<<1, DESC_CHUNK, 0, s>>>(d + i, c);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
 // B reversed into temp for the window kernel, whose bulk copies need B
 // stored descending (element y of B at out[nb-1-y])
 __global__ void reverse_u32_kernel(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, long long n) {
@@ -717,7 +739,7 @@ static bcf_status merge_runs_impl(const uint32_t* d_runs, const uint32_t* const*
       next.push_back(o);
     }
     GroupDesc* dt = dtab + (size_t)(i - 1) * (table_bytes / sizeof(GroupDesc));
-    cudaError_t e = cudaMemcpyAsync(dt, tab.data(), tab.size() * sizeof(GroupDesc), cudaMemcpyHostToDevice, s);
+    cudaError_t e = write_table(dt, tab, s);  // kernel launches: capturable into a CUDA graph
     if (e != cudaSuccess) return cuda_fail(e);
     MergeArgs ma{srck, srcv, dk, dv, (long long)n, 0, 0, 0, 0, dt, (int)tab.size(), nullptr};
     if (i == 1 && rev1) {

@@ -556,3 +556,27 @@ print("even-window ok")
     env = dict(os.environ, BCF_EVEN_WIN="1")
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "even-window ok" in r.stdout, r.stdout + r.stderr
+
+
+def test_cuda_graph_capture_merge_runs():
+    """bcf_merge_runs_u32 (the distributed sort's final merge) writes its
+    per-pass descriptor tables with small kernels, so it can be captured into
+    a CUDA graph; each replay re-merges the current run contents."""
+    sizes = [30001, 29999, 12345, 50000, 7, 25000]
+    offs = np.concatenate([[0], np.cumsum(sizes)]).astype(np.uint64)
+    def runs_for(seed):
+        return np.concatenate([np.sort(si.uniform_u32(m, seed + i)) for i, m in enumerate(sizes)])
+    r0 = runs_for(31)
+    runs = to_dev(r0)
+    out0 = bcf.merge_runs(runs, offs)  # warm-up outside the capture (attribute caches)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(to_host(out0), oracle.sort_u32(r0))
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        out = bcf.merge_runs(runs, offs)
+    for seed in (41, 42):
+        rs = runs_for(seed)
+        runs.copy_(to_dev(rs))
+        g.replay()
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(to_host(out), oracle.sort_u32(rs))
