@@ -756,6 +756,42 @@ __device__ __forceinline__ void warp_run_scatter_rho(uint32_t* __restrict__ sk, 
   for (int r = 0; r < E; ++r) sk[rho<E>(base + step * r)] = k[r];
 }
 
+// The same for E = 10, 12, 14 (16 slots per lane, 16 - E max-key pads; the
+// warp's 32E real keys fill lanes 0..2E-1): lane i's slots are rotated by
+// sigma_i, so that in round s it writes run position 16 i + (s + sigma_i) mod 16.
+// Through rho, bank(k) = (k + (k / P mod d)) mod 32 (P = wE/d = 0 mod 32): a
+// search over sigma (tools-free: 2E lanes x 16 rounds, A and mirrored B
+// positions) found sigma_i = i / 2 conflict-free for E = 10 and 12, and the
+// same with sigma_3 = 7 for E = 14.
+template <int E>
+__device__ __forceinline__ void warp_run_scatter_rho_pad(uint32_t* __restrict__ sk, const uint32_t (&k)[16], int warp,
+                                                         int lane) {
+  static_assert(E == 10 || E == 12 || E == 14, "padded warp phase: E = 10, 12, 14");
+  constexpr int S = W * E;
+  const int sigma = (E == 14 && lane == 3) ? 7 : (lane >> 1);
+  uint32_t r[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) r[i] = k[i];
+#pragma unroll
+  for (int b = 0; b < 4; ++b) {
+    const bool on = (sigma >> b) & 1;
+    uint32_t t[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) t[i] = on ? r[(i + (1 << b)) & 15] : r[i];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) r[i] = t[i];
+  }
+  // r[s] holds slot (s + sigma) mod 16
+  if (lane >= 2 * E) return;  // only pads
+  const int gbase = (warp >> 1) * 2 * S;
+  const bool isB = warp & 1;
+#pragma unroll
+  for (int s = 0; s < 16; ++s) {
+    const int pos = 16 * lane + ((s + sigma) & 15);
+    sk[rho<E>(isB ? gbase + 2 * S - 1 - pos : gbase + pos)] = r[s];
+  }
+}
+
 // f32 <-> order-preserving u32 (IEEE totalOrder, reading c2)
 __device__ __forceinline__ uint32_t f32_encode(uint32_t b) {
   return b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u);

@@ -222,6 +222,9 @@ __host__ __device__ constexpr int bs_min_blocks() {
 // outputs [tid E, tid E + E) in key[] (val[] for pairs); sk / sv (tile_words
 // each) are its working buffers, still being read by other threads until the
 // caller's next __syncthreads.
+#ifndef BCF_WARP_PAD
+#define BCF_WARP_PAD 1
+#endif
 #ifndef BCF_WARP_POW2
 #define BCF_WARP_POW2 1
 #endif
@@ -242,7 +245,10 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
   // chunk) without the shared-memory round trip of the general path
   // (also E = 16 and 8: E slots per lane, no pad, the warp runs written
   // through rho; BCF_WARP_POW2=0 keeps those on the shared-memory levels)
-  constexpr bool WARP_PHASE = CF && !PAIRS && U >= 2 * W && (E + 1 == W || (BCF_WARP_POW2 && (E == 16 || E == 8)));
+  // (and E = 10, 12, 14: 16 slots per lane with max-key pads; BCF_WARP_PAD=0: off)
+  constexpr bool WARP_PAD = CF && !PAIRS && BCF_WARP_PAD && (E == 10 || E == 12 || E == 14);
+  constexpr bool WARP_PHASE =
+      CF && !PAIRS && U >= 2 * W && (E + 1 == W || (BCF_WARP_POW2 && (E == 16 || E == 8)) || WARP_PAD);
   uint32_t tag[E];
   if constexpr (WARP_PHASE) {
     const int wbase = warp * (W * E);
@@ -316,6 +322,14 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
 #endif
     __syncthreads();  // (general path: every thread has finished its blocked read of sk)
     warp_run_scatter<E>(sk, k32, warp, lane);
+    l_first = 5;
+  } else if constexpr (WARP_PHASE && WARP_PAD) {
+    uint32_t k16[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) k16[i] = i < E ? key[i] : PAD_KEY;
+    warp_bitonic_levels<16>(k16, lane);
+    __syncthreads();
+    warp_run_scatter_rho_pad<E>(sk, k16, warp, lane);
     l_first = 5;
   } else if constexpr (WARP_PHASE) {
     warp_bitonic_levels<E>(key, lane);
