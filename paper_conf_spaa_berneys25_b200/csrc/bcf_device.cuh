@@ -756,17 +756,18 @@ __device__ __forceinline__ void warp_run_scatter_rho(uint32_t* __restrict__ sk, 
   for (int r = 0; r < E; ++r) sk[rho<E>(base + step * r)] = k[r];
 }
 
-// The same for E = 10, 12, 14 (16 slots per lane, 16 - E max-key pads; the
+// The same for E < 16 other than 8 (16 slots per lane, 16 - E max-key pads; the
 // warp's 32E real keys fill lanes 0..2E-1): lane i's slots are rotated by
 // sigma_i, so that in round s it writes run position 16 i + (s + sigma_i) mod 16.
 // Through rho, bank(k) = (k + (k / P mod d)) mod 32 (P = wE/d = 0 mod 32): a
-// search over sigma (tools-free: 2E lanes x 16 rounds, A and mirrored B
-// positions) found sigma_i = i / 2 conflict-free for E = 10 and 12, and the
-// same with sigma_3 = 7 for E = 14.
+// search over sigma (2E lanes x 16 rounds, A and mirrored B positions) found
+// sigma_i = i / 2 conflict-free for E = 10 and 12, and the same with
+// sigma_3 = 7 for E = 14; for odd E (rho = identity) sigma_i = i / 2 gives the
+// banks 16 (i mod 2) + (s + i / 2) mod 16, distinct for 2E <= 30 lanes.
 template <int E>
 __device__ __forceinline__ void warp_run_scatter_rho_pad(uint32_t* __restrict__ sk, const uint32_t (&k)[16], int warp,
                                                          int lane) {
-  static_assert(E == 10 || E == 12 || E == 14, "padded warp phase: E = 10, 12, 14");
+  static_assert(E <= 15 && E != 8, "padded warp phase: E < 16 (E = 8 has no pads)");
   constexpr int S = W * E;
   const int sigma = (E == 14 && lane == 3) ? 7 : (lane >> 1);
   uint32_t r[16];

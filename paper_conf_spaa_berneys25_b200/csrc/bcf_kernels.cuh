@@ -245,8 +245,8 @@ __device__ __forceinline__ void block_sort_core(const SortArgs& args, uint32_t* 
   // chunk) without the shared-memory round trip of the general path
   // (also E = 16 and 8: E slots per lane, no pad, the warp runs written
   // through rho; BCF_WARP_POW2=0 keeps those on the shared-memory levels)
-  // (and E = 10, 12, 14: 16 slots per lane with max-key pads; BCF_WARP_PAD=0: off)
-  constexpr bool WARP_PAD = CF && !PAIRS && BCF_WARP_PAD && (E == 10 || E == 12 || E == 14);
+  // (and E < 16 other than 8: 16 slots per lane with max-key pads; BCF_WARP_PAD=0: off)
+  constexpr bool WARP_PAD = CF && !PAIRS && BCF_WARP_PAD && E < 16 && E != 8;
   constexpr bool WARP_PHASE =
       CF && !PAIRS && U >= 2 * W && (E + 1 == W || (BCF_WARP_POW2 && (E == 16 || E == 8)) || WARP_PAD);
   uint32_t tag[E];
